@@ -1,0 +1,260 @@
+"""TEST INFRASTRUCTURE -- Python face of the fp64 CPU oracle (bvh_oracle.cpp).
+
+Only tests/, __graft_entry__.smoke() and bench.py (cpu_baseline leg and
+``--impl reference``) may import this module.  It shares no code with the
+CUDA path.  Citations: P:NNN = line of /root/reference/PAPER.md; [A#] =
+reading in DESIGN.md.
+
+``step()`` composes Alg. 6 from the C++ pieces:
+bbox -> keys -> stable sort -> permute -> build -> force -> leapfrog (O8).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+import time
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "bvh_oracle.cpp")
+_LIB = os.path.join(_HERE, "libbvh_oracle.so")
+_lib = None
+
+_P = C.c_void_p
+_f32p = np.ctypeslib.ndpointer(np.float32, flags="C_CONTIGUOUS")
+_f64p = np.ctypeslib.ndpointer(np.float64, flags="C_CONTIGUOUS")
+_u32p = np.ctypeslib.ndpointer(np.uint32, flags="C_CONTIGUOUS")
+_u64p = np.ctypeslib.ndpointer(np.uint64, flags="C_CONTIGUOUS")
+_i64p = np.ctypeslib.ndpointer(np.int64, flags="C_CONTIGUOUS")
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle (plain g++, no fast-math, no contraction)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
+               "-pthread", "-o", _LIB + ".tmp", _SRC]
+        subprocess.run(cmd, check=True)
+        os.replace(_LIB + ".tmp", _LIB)
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        L = C.CDLL(build())
+        L.orc_paper_key_bits.argtypes = [C.c_int64]
+        L.orc_paper_key_bits.restype = C.c_int
+        L.orc_hilbert_index.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, C.c_int]
+        L.orc_hilbert_index.restype = C.c_uint64
+        L.orc_bbox.argtypes = [C.c_int64, _f32p, _f32p, _f32p]
+        L.orc_quantize.argtypes = [C.c_int64, _f32p, _f32p, _f32p, C.c_int, _u32p]
+        L.orc_keys.argtypes = [C.c_int64, _f32p, C.c_int, _u64p]
+        L.orc_sort.argtypes = [C.c_int64, _u64p, _u32p]
+        L.orc_build.argtypes = [C.c_int64, _f32p, _f32p]
+        L.orc_build.restype = _P
+        L.orc_free_tree.argtypes = [_P]
+        L.orc_free_tree.restype = None
+        L.orc_tree_levels.argtypes = [_P]
+        L.orc_tree_count.argtypes = [_P, C.c_int]
+        L.orc_tree_count.restype = C.c_int64
+        L.orc_tree_level.argtypes = [_P, C.c_int, _P, _P, _P, _P, _P]
+        L.orc_force.argtypes = [_P, C.c_double, C.c_double, _i64p, C.c_int64, _f64p, _P, C.c_int]
+        L.orc_force_list.argtypes = [_P, C.c_double, C.c_double, C.c_int64, _i64p, C.c_int64]
+        L.orc_force_list.restype = C.c_int64
+        L.orc_direct.argtypes = [C.c_int64, _f32p, _f32p, C.c_double, _i64p, C.c_int64, _f64p, C.c_int]
+        for f in ("orc_bbox", "orc_quantize", "orc_keys", "orc_sort", "orc_tree_levels", "orc_tree_level",
+                  "orc_force", "orc_direct"):
+            getattr(L, f).restype = C.c_int
+        _lib = L
+    return _lib
+
+
+def _ok(rc: int, what: str):
+    if rc != 0:
+        raise ValueError(f"oracle {what} failed (rc={rc})")
+
+
+def _f32(a, shape=None):
+    a = np.ascontiguousarray(a, np.float32)
+    if shape is not None:
+        a = a.reshape(shape)
+    return a
+
+
+# ------------------------------------------------------------------ O1..O4 --
+def paper_key_bits(n: int) -> int:
+    """[A8] smallest b >= 1 with 8^b >= N."""
+    return lib().orc_paper_key_bits(int(n))
+
+
+def resolve_key_bits(n: int, key_bits: int) -> int:
+    return paper_key_bits(n) if key_bits == 0 else int(key_bits)
+
+
+def hilbert_index(x: int, y: int, z: int, b: int) -> int:
+    """Skilling's transpose + MSB-first interleave (ref [17])."""
+    return int(lib().orc_hilbert_index(x, y, z, b))
+
+
+def bbox(pos):
+    """O1 -- Alg. 3."""
+    pos = _f32(pos, (-1, 3))
+    lo = np.empty(3, np.float32)
+    hi = np.empty(3, np.float32)
+    _ok(lib().orc_bbox(len(pos), pos, lo, hi), "bbox")
+    return lo, hi
+
+
+def quantize(pos, b: int):
+    """O2 -- grid cells [A9][A17]."""
+    pos = _f32(pos, (-1, 3))
+    lo, hi = bbox(pos)
+    q = np.empty((len(pos), 3), np.uint32)
+    _ok(lib().orc_quantize(len(pos), pos, lo, hi, int(b), q), "quantize")
+    return q
+
+
+def keys(pos, b: int):
+    """O1..O3 -- Hilbert key per body in current slot order."""
+    pos = _f32(pos, (-1, 3))
+    out = np.empty(len(pos), np.uint64)
+    _ok(lib().orc_keys(len(pos), pos, int(b), out), "keys")
+    return out
+
+
+def sort_perm(k):
+    """O4 -- stable sort; perm[k] = current slot of the body now at slot k."""
+    k = np.ascontiguousarray(k, np.uint64)
+    perm = np.empty(len(k), np.uint32)
+    _ok(lib().orc_sort(len(k), k, perm), "sort")
+    return perm
+
+
+# --------------------------------------------------------------------- O6 --
+@dataclass
+class LevelData:
+    M: np.ndarray      # fp64 [c]
+    com: np.ndarray    # fp64 [c,3]
+    s2: np.ndarray     # fp64 [c]
+    lo: np.ndarray     # fp32 [c,3]
+    hi: np.ndarray     # fp32 [c,3]
+
+    @property
+    def m32(self):
+        return self.M.astype(np.float32)
+
+    @property
+    def c32(self):
+        return self.com.astype(np.float32)
+
+
+class Tree:
+    """O6 -- BUILDTREEACCUMULATEMASS over Hilbert-sorted bodies."""
+
+    def __init__(self, pos_sorted, mass_sorted):
+        self.pos = _f32(pos_sorted, (-1, 3))
+        self.mass = _f32(mass_sorted, (-1,))
+        if len(self.pos) != len(self.mass) or len(self.pos) < 1:
+            raise ValueError("bad tree input")
+        self.n = len(self.pos)
+        self._h = lib().orc_build(self.n, self.pos, self.mass)
+        if not self._h:
+            raise MemoryError("orc_build failed")
+        self.L = lib().orc_tree_levels(self._h)
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h and _lib is not None:
+            _lib.orc_free_tree(h)
+            self._h = None
+
+    def count(self, level: int) -> int:
+        return int(lib().orc_tree_count(self._h, level))
+
+    def level(self, l: int) -> LevelData:
+        c = self.count(l)
+        if c < 0:
+            raise IndexError(l)
+        d = LevelData(np.empty(c), np.empty((c, 3)), np.empty(c), np.empty((c, 3), np.float32),
+                      np.empty((c, 3), np.float32))
+        _ok(lib().orc_tree_level(self._h, l, d.M.ctypes.data, d.com.ctypes.data, d.s2.ctypes.data,
+                                 d.lo.ctypes.data, d.hi.ctypes.data), "tree_level")
+        return d
+
+    def force(self, theta: float, eps: float, targets=None, nthreads: int = 0):
+        """O7 -- per-target DFS; returns (acc fp64 [nt,3], interactions int64 [nt])."""
+        t = np.arange(self.n, dtype=np.int64) if targets is None else np.ascontiguousarray(targets, np.int64)
+        acc = np.empty((len(t), 3))
+        cnt = np.empty(len(t), np.int64)
+        _ok(lib().orc_force(self._h, float(theta), float(eps), t, len(t), acc, cnt.ctypes.data, int(nthreads)),
+            "force")
+        return acc, cnt
+
+    def force_list(self, theta: float, eps: float, target: int):
+        """O7 interaction list of one target: int64 [len, 2] of (level, index), DFS order."""
+        cap = 4 * self.n + 64
+        out = np.empty(2 * cap, np.int64)
+        c = lib().orc_force_list(self._h, float(theta), float(eps), int(target), out, cap)
+        if c < 0:
+            raise ValueError("force_list failed")
+        return out[: 2 * c].reshape(c, 2)
+
+
+def direct(pos, mass, eps: float, targets=None, nthreads: int = 0):
+    """D -- direct summation of Eq. 1, softened, fp64."""
+    pos = _f32(pos, (-1, 3))
+    mass = _f32(mass, (-1,))
+    t = np.arange(len(pos), dtype=np.int64) if targets is None else np.ascontiguousarray(targets, np.int64)
+    acc = np.empty((len(t), 3))
+    _ok(lib().orc_direct(len(pos), pos, mass, float(eps), t, len(t), acc, int(nthreads)), "direct")
+    return acc
+
+
+# ------------------------------------------------------------- the step ---
+@dataclass
+class StepResult:
+    keys: np.ndarray        # u64 [n], pre-sort slot order
+    perm: np.ndarray        # u32 [n]: sorted slot k <- previous slot perm[k]
+    tree: Tree
+    acc: np.ndarray         # fp64 [nt,3] for `targets` (sorted slots)
+    count: np.ndarray       # int64 [nt]
+    targets: np.ndarray     # sorted slots the force was evaluated for
+    pos: np.ndarray         # fp32 [n,3] sorted, after the update (if integrated)
+    vel: np.ndarray         # fp32 [n,3] sorted, after the update
+    mass: np.ndarray        # fp32 [n] sorted
+    ids: np.ndarray         # int64 [n]: body id in each sorted slot
+    seconds: float
+
+
+def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_bits: int = 16,
+         integrate: bool = True, targets=None, nthreads: int = 0) -> StepResult:
+    """One step of Alg. 6 on fp32 state in the current slot order.
+
+    O8 [A14] kick-drift leapfrog, v_{+1/2} = v_{-1/2} + a dt, x += v_{+1/2} dt,
+    evaluated in fp64 and stored in fp32 (the state precision of the path).
+    With ``targets`` (sorted slots) only those bodies get forces and the
+    update is skipped.
+    """
+    t0 = time.perf_counter()
+    pos = _f32(pos, (-1, 3))
+    vel = _f32(vel, (-1, 3))
+    mass = _f32(mass, (-1,))
+    n = len(pos)
+    ids = np.arange(n, dtype=np.int64) if ids is None else np.asarray(ids, np.int64)
+    b = resolve_key_bits(n, key_bits)
+    k = keys(pos, b)                           # O1-O3
+    perm = sort_perm(k)                        # O4
+    ps, vs, ms, ids_s = pos[perm], vel[perm], mass[perm], ids[perm]  # O5 [A11]
+    tree = Tree(ps, ms)                        # O6
+    full = targets is None
+    tg = np.arange(n, dtype=np.int64) if full else np.ascontiguousarray(targets, np.int64)
+    acc, cnt = tree.force(theta, eps, tg, nthreads)   # O7
+    if integrate and full:                     # O8
+        v_new = vs.astype(np.float64) + acc * dt
+        x_new = ps.astype(np.float64) + v_new * dt
+        vs = v_new.astype(np.float32)
+        ps = x_new.astype(np.float32)
+    return StepResult(k, perm, tree, acc, cnt, tg, ps, vs, ms, ids_s, time.perf_counter() - t0)
