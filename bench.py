@@ -1,0 +1,328 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 Hilbert-BVH Barnes-Hut step (BASELINE.json metric:
+"BH step time & bodies/s (theta=0.5, N=10M) at 1/2/4/8 B200; interactions/s").
+
+Workload: config 3 of BASELINE.json -- two-disk galaxy collision, N = 10^7,
+theta = 0.5, eps = 1e-3, dt = 1e-3, fixed 16-bit Hilbert grid (DESIGN.md
+A8), synthetic seeded input (workloads/).  A "step" is one full pass of
+Alg. 6: bbox, keys, radix sort, permute, build, force, leapfrog.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Prints one JSON line (rank 0).  For N > 1 launch with torch.distributed.run.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from workloads import CONFIGS, generate  # noqa: E402
+
+FLOPS_PER_INTERACTION = 20  # 3 sub + 3 mul/fma (r^2) + eps add + rsqrt + 3 mul + 3 fma ~ 20 flop
+METRIC = "BH step bodies/s (theta=0.5, N=10M)"
+UNIT = "bodies/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="cfg3")
+    ap.add_argument("--n", type=int, default=0, help="override N (testing only)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target oracle force-sample time")
+    return ap.parse_args()
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def workload(args):
+    cfg = dict(CONFIGS[args.config])
+    if args.n:
+        cfg["n"] = args.n
+    return cfg
+
+
+def config_json(cfg, world, extra=None):
+    d = {"workload": f"{cfg['workload']} N={cfg['n']} ({args_config_name(cfg)})", "n": cfg["n"],
+         "theta": cfg["theta"], "eps": cfg["eps"], "dt": cfg["dt"], "key_bits": 16, "seed": cfg["seed"],
+         "parallelism": "single" if world == 1 else f"hilbert-range x{world}",
+         "l2": "inputs larger than L2 (bodies 320 MB + tree ~1 GB per step at N=1e7); no explicit flush"}
+    if extra:
+        d.update(extra)
+    return d
+
+
+def args_config_name(cfg):
+    for k, v in CONFIGS.items():
+        if v["workload"] == cfg["workload"] and v["seed"] == cfg["seed"]:
+            return k
+    return "custom"
+
+
+# ------------------------------------------------------------- clocks ------
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.p = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                       "-lms", "50", "-i", str(self.idx)], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        rows = [[x.strip() for x in ln.split(",")] for ln in out.strip().splitlines() if ln.count(",") >= 8]
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        smax = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": reasons, "samples": len(rows),
+                "power_w_max": max((float(r[3]) for r in rows if r[3].replace(".", "").isdigit()), default=None)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def ncu_traffic():
+    """dram bytes per launch of the force kernel from the committed ncu
+    --set full capture summary (profiles/*force_ncu.json), or None."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*force_ncu*.json")))
+    if not files:
+        return None
+    try:
+        with open(files[-1]) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+# ----------------------------------------------------------- CPU oracle ----
+def cpu_oracle_sample(pos, vel, mass, cfg, target_seconds, seed=0):
+    """Oracle step on the full input with forces for a bounded random sample
+    of targets; returns (bodies/s extrapolated to all N, description, cores,
+    interactions/s)."""
+    from oracle import oracle as O
+    n = len(pos)
+    rng = np.random.default_rng(seed)
+    probe = np.sort(rng.choice(n, min(n, 500), replace=False))
+    t0 = time.perf_counter()
+    r = O.step(pos, vel, mass, theta=cfg["theta"], eps=cfg["eps"], dt=cfg["dt"], key_bits=16, integrate=False,
+               targets=probe)
+    t_all = time.perf_counter() - t0
+    tf0 = time.perf_counter()
+    r.tree.force(cfg["theta"], cfg["eps"], probe)
+    t_probe = time.perf_counter() - tf0
+    t_prep = max(0.0, t_all - t_probe)
+    per_target = max(t_probe / len(probe), 1e-9)
+    ns = int(min(n, max(len(probe), target_seconds / per_target)))
+    targets = np.sort(rng.choice(n, ns, replace=False))
+    tf0 = time.perf_counter()
+    _, cnt = r.tree.force(cfg["theta"], cfg["eps"], targets)
+    t_force = time.perf_counter() - tf0
+    t_full = t_prep + t_force * n / ns
+    cores = os.cpu_count()
+    desc = (f"oracle (fp64 C++, g++ -O2, {cores} threads) full bbox/keys/stable-sort/permute/build on N={n}, "
+            f"forces for {ns} random targets ({t_force:.1f} s), extrapolated to all N; prep {t_prep:.1f} s")
+    return n / t_full, desc, cores, float(cnt.sum()) / t_force, t_full
+
+
+# ------------------------------------------------------------ reference ----
+def run_reference(args, cfg, world, rank):
+    if rank != 0:
+        return 0
+    pos, vel, mass = generate(cfg["workload"], cfg["n"], cfg["seed"])
+    times = []
+    desc = cores = ips = None
+    for i in range(args.warmup + args.steps):
+        v, desc, cores, ips, t_full = cpu_oracle_sample(pos, vel, mass, cfg, min(args.cpu_seconds, 6.0), seed=i)
+        if i >= args.warmup:
+            times.append(t_full)
+    ms = 1e3 * statistics.mean(times)
+    value = cfg["n"] / (ms / 1e3)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": config_json(cfg, 1),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc,
+                             "interactions_per_s": ips},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ ours ----
+def run_ours(args, cfg, world, rank, local):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_casselldahg24_b200 import NBody
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n = cfg["n"]
+    pos, vel, mass = generate(cfg["workload"], n, cfg["seed"])
+    stream = torch.cuda.Stream()
+    sim = NBody(n, cfg["theta"], cfg["eps"], cfg["dt"], key_bits=16, stream=stream.cuda_stream)
+    if world > 1:
+        sim.attach_process_group(rank, world)
+    sim.set_bodies(pos, vel, mass)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    sim.step(args.warmup)
+    barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    sim.step(args.steps)
+    e1.record(stream)
+    barrier()
+    ms_total = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    if world > 1:
+        t = torch.tensor([ms_total], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms = ms_total / args.steps
+    st = sim.stats()
+    inter = int(st["interactions"])  # last step, owned targets of this rank
+    if world > 1:
+        t = torch.tensor([inter], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t)
+        inter = int(t.item())
+    launches = int(st["kernels_per_step"]) * args.steps
+
+    # Dominant kernel (K6 force): its device time per launch, measured live
+    # with CUDA events on the launching stream, graphs off.
+    sim.set_option(5, 1)  # NBODY_OPT_TIMING
+    sim.set_option(3, 0)  # NBODY_OPT_USE_GRAPH
+    f_ms, f_int, stage = [], [], {}
+    for _ in range(max(3, min(args.steps, 5))):
+        sim.step(1)
+        s2 = sim.stats()
+        f_ms.append(s2["ms_force"])
+        f_int.append(s2["interactions"])
+        for k in ("ms_bbox_keys", "ms_sort", "ms_build", "ms_force", "ms_update"):
+            stage.setdefault(k, []).append(s2[k])
+    sim.set_option(3, 1)
+    sim.set_option(5, 0)
+    force_ms = statistics.mean(f_ms)
+    force_flops = FLOPS_PER_INTERACTION * statistics.mean(f_int)
+    peaks = measured_peaks()
+    nsm = torch.cuda.get_device_properties(local).multi_processor_count
+    fmax = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_tflops = 2 * 128 * nsm * fmax * 1e6 / 1e12  # FP32 FFMA lanes x 2 flop x SMs x max clock
+    achieved = force_flops / (force_ms / 1e3) / 1e12
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
+                "frac": achieved / peak_tflops, "traffic": ncu_traffic(),
+                "kernel": "k_force (CALCULATEFORCE)", "flops_per_interaction": FLOPS_PER_INTERACTION,
+                "kernel_ms": force_ms,
+                "peak_basis": f"FP32 pipe 2 flop x 128 lanes x {nsm} SMs x {fmax:.0f} MHz (sm_max, MEASURED_PEAKS.json)",
+                "share_of_step": force_ms / ms}
+
+    # End to end through the public API: pinned host inputs -> step -> host result.
+    e2e = None
+    if not args.no_e2e:
+        hp = torch.from_numpy(pos).pin_memory()
+        hv = torch.from_numpy(vel).pin_memory()
+        hm = torch.from_numpy(mass).pin_memory()
+        out = torch.empty((n, 3), dtype=torch.float32).pin_memory()
+        if world == 1:
+            sim.set_bodies(hp, hv, hm)
+            sim.step(1)
+            sim.get_positions(out)
+            barrier()
+            t0 = time.perf_counter()
+            for _ in range(args.steps):
+                sim.set_bodies(hp, hv, hm)
+                sim.step(1)
+                sim.get_positions(out)
+            barrier()
+            e2e_ms = 1e3 * (time.perf_counter() - t0) / args.steps
+            e2e = {"value": n / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": 28 * n,
+                   "d2h_bytes_per_step": 12 * n, "ms_per_step": e2e_ms,
+                   "path": "nbody_set_bodies(pinned host) + nbody_step(1) + nbody_get_positions(pinned host)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, desc, cores, ips, _ = cpu_oracle_sample(pos, vel, mass, cfg, args.cpu_seconds)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc,
+               "interactions_per_s": ips}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "f32 (fp64 tree moments, key grid and opening test)",
+                "data": "synthetic", "impl": "ours",
+                "config": config_json(cfg, world),
+                "interactions_per_s": inter / (ms / 1e3), "interactions_per_body": inter / n,
+                "stage_ms": {k: statistics.mean(v) for k, v in stage.items()},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                "clocks": clk}
+        print(json.dumps(line), flush=True)
+    sim.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    world, rank, local = dist_env()
+    cfg = workload(args)
+    if args.impl == "reference":
+        return run_reference(args, cfg, world, rank)
+    return run_ours(args, cfg, world, rank, local)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

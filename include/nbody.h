@@ -1,0 +1,163 @@
+/*
+ * nbody.h -- C ABI of the B200-native Hilbert-sorted BVH Barnes-Hut step.
+ *
+ * Method: Cassell, Deakin, Alpay, Heuveline, Brito Gadeschi, "Efficient
+ * Tree-based Parallel Algorithms for N-Body Simulations Using C++ Standard
+ * Parallelism", SC'24.  P:NNN below = line NNN of the paper text
+ * (/root/reference/PAPER.md); [A#] = a reading of the paper listed in
+ * DESIGN.md "Readings".
+ *
+ * One time step is Alg. 6:
+ *   CALCULATEBOUNDINGBOX (Alg. 3) -> HILBERTSORT (Alg. 7,
+ *   P:201-212) -> BUILDTREEACCUMULATEMASS (P:218, P:221,
+ *   Fig. 4) -> CALCULATEFORCE (Eq. 1
+ *   P:72) -> UPDATEPOSITION (Stormer-Verlet).
+ * Every stage runs in hand-written sm_100a CUDA kernels of this library.
+ *
+ * Conventions (all functions):
+ *   - G = 1 [A2].  Softened gravity a_i = sum_j m_j r_ij / (|r_ij|^2 + eps^2)^(3/2) [A1].
+ *   - Bodies live in "slots".  Slot order is the caller's array order until
+ *     the first force pass; afterwards it is the Hilbert order of the last
+ *     sort (each step re-sorts the previous step's order).  The body id is
+ *     the index in the arrays passed to nbody_set_bodies and travels with
+ *     the body.  Functions documented "by id" return arrays indexed by id.
+ *   - Pointers to caller buffers may be host (pageable or pinned) or device
+ *     pointers of the context's device; the library detects which.  The
+ *     caller owns every buffer it passes; the library never keeps a caller
+ *     pointer past the call.  Calls that read results synchronise the
+ *     context's stream; nbody_step / nbody_compute_accel are asynchronous.
+ *   - Not thread-safe per context; one context per (device, stream).
+ *   - Every function returns NBODY_OK or a negative status.  No C++
+ *     exception or abort crosses the ABI.  After a CUDA failure the context
+ *     is in NBODY_ESTATE until nbody_destroy; nbody_last_error() explains.
+ */
+#ifndef NBODY_B200_H
+#define NBODY_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct nbody_ctx nbody_ctx; /* opaque, owned by the library */
+
+typedef enum {
+  NBODY_OK = 0,
+  NBODY_EINVAL = -1, /* bad argument (null, range, non-finite input)      */
+  NBODY_ENOMEM = -2, /* device allocation failed                          */
+  NBODY_ECUDA = -3,  /* CUDA error; context now in NBODY_ESTATE           */
+  NBODY_ENCCL = -4,  /* NCCL error; context now in NBODY_ESTATE           */
+  NBODY_ESTATE = -5  /* call not valid in the current state               */
+} nbody_status;
+
+/* Options for nbody_set_option. */
+enum {
+  /* Hilbert grid bits per axis b [A8]: 0 = the paper's count rule
+   * (smallest b with 8^b >= N); 1..21 = fixed b.  Default 16.  Keys hold
+   * 3b bits; b <= 10 sorts 32-bit keys, b >= 11 64-bit keys.  Must be set
+   * before nbody_set_bodies. */
+  NBODY_OPT_KEY_BITS = 1,
+  /* cudaStream_t (cast to int64) all work is issued on; 0 = the library's
+   * own non-blocking stream (default). */
+  NBODY_OPT_STREAM = 2,
+  /* 1 = capture one step in a CUDA graph and replay it (default), 0 = plain
+   * launches. */
+  NBODY_OPT_USE_GRAPH = 3,
+  /* CALCULATEFORCE kernel variant: 0 = default (fastest validated),
+   * 1 = warp mask-stack walk (per-lane exact lists, no group lists). */
+  NBODY_OPT_TRAVERSAL = 4,
+  /* 1 = record CUDA events around each stage of a pass issued by
+   * nbody_compute_accel / nbody_step with graphs off; nbody_get_stats then
+   * reports the device time of each stage of the last pass.  Default 0. */
+  NBODY_OPT_TIMING = 5
+};
+
+typedef struct {
+  int64_t n;                  /* bodies                                   */
+  int key_bits;               /* resolved b                               */
+  int levels;                 /* L = ceil(log2 N) levels above the leaves */
+  int64_t steps;              /* force passes done since set_bodies       */
+  uint64_t interactions;      /* interactions of the last force pass, summed over owned targets */
+  float ms_bbox_keys;         /* per-stage device time of the last pass   */
+  float ms_sort;              /* (valid only when graphs are off and      */
+  float ms_build;             /*  NBODY_OPT_TIMING is on; else 0):        */
+  float ms_force;             /*  K1+K2, K3, K4+K5, K6, K7                */
+  float ms_update;
+  int kernels_per_step;       /* library kernel launches in one step      */
+} nbody_stats;
+
+/* Library version (major*10000 + minor*100 + patch). */
+int nbody_version(void);
+
+/* Create a context for n bodies on the current CUDA device.
+ *   n in [1, 2^30 - 1] (the sort packs counts in 30 bits); theta >= 0 (opening parameter, accept a node iff
+ *   s^2 < theta^2 d^2, [A3]); eps >= 0 (Plummer softening [A1]); dt finite
+ *   (leapfrog step [A14]).  All device memory is allocated here (tree
+ *   sizes are fixed by N).  *out is set to NULL on failure. */
+nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx **out);
+
+/* Set an option (see enum).  Returns NBODY_EINVAL for an unknown option or
+ * value, NBODY_ESTATE if the option can no longer change. */
+nbody_status nbody_set_option(nbody_ctx *ctx, int option, int64_t value);
+
+/* Load the bodies: pos[n][3], vel[n][3] (read as v_{-1/2} [A14]), mass[n],
+ * fp32, host or device.  Copies them; resets slot order to array order and
+ * ids to array indices.  Masses must be > 0 and finite, positions and
+ * velocities finite [A18]. */
+nbody_status nbody_set_bodies(nbody_ctx *ctx, const float *pos, const float *vel, const float *mass);
+
+/* Stages 1-5 of Alg. 6 at the current positions (no UPDATEPOSITION):
+ * bbox, keys, sort, permute, build, force.  Afterwards slot order is the
+ * new Hilbert order and nbody_get_accel returns a(x_t).  Asynchronous. */
+nbody_status nbody_compute_accel(nbody_ctx *ctx);
+
+/* nsteps full steps of Alg. 6 (force pass + kick-drift leapfrog
+ * v += a dt, x += v dt [A14]).  Asynchronous on the context stream. */
+nbody_status nbody_step(nbody_ctx *ctx, int nsteps);
+
+/* Wait for all work issued on the context stream. */
+nbody_status nbody_sync(nbody_ctx *ctx);
+
+/* a(x) of the last force pass, out[n][3] by id (fp32). */
+nbody_status nbody_get_accel(nbody_ctx *ctx, float *out);
+
+/* Current positions / velocities, out[n][3] by id (fp32). */
+nbody_status nbody_get_positions(nbody_ctx *ctx, float *out);
+nbody_status nbody_get_velocities(nbody_ctx *ctx, float *out);
+
+/* Interactions per body of the last force pass, out[n] by id. */
+nbody_status nbody_get_interactions(nbody_ctx *ctx, uint32_t *out);
+
+/* Full state in slot order: pos_m[n][4] = (x, y, z, m), vel_id[n][4] =
+ * (vx, vy, vz, id reinterpreted as float bits). */
+nbody_status nbody_get_state(nbody_ctx *ctx, float *pos_m, float *vel_id);
+
+nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
+
+/* ---- debug views of the last force pass (parity tests) ---------------- */
+/* Hilbert keys of the bodies in the slot order BEFORE the last sort:
+ * keys[n] as uint64 (3b bits, Skilling's index). */
+nbody_status nbody_debug_keys(nbody_ctx *ctx, uint64_t *keys);
+/* Sort permutation: sorted slot k <- previous slot perm[k] (stable [A10]). */
+nbody_status nbody_debug_perm(nbody_ctx *ctx, uint32_t *perm);
+/* Level l in [1, L] of the BVH: *count = ceil(N / 2^l) nodes;
+ * pred[count][4] fp64 = (com_x, com_y, com_z, s^2) (the opening-test data,
+ * com = sum(m x) / sum(m) in fp64, s = longest AABB side [A3]);
+ * rec[count][4] fp32 = ((float)com, (float)M) (the monopole used in the
+ * interaction); box[count][6] fp32 = (lo xyz, hi xyz).  Any of pred, rec,
+ * box may be NULL; pass all NULL to query *count. */
+nbody_status nbody_debug_level(nbody_ctx *ctx, int level, int64_t *count, double *pred, float *rec, float *box);
+
+/* Human-readable description of the last error on this context (never NULL). */
+const char *nbody_last_error(const nbody_ctx *ctx);
+
+/* Free all resources.  NULL is a no-op. */
+void nbody_destroy(nbody_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* NBODY_B200_H */

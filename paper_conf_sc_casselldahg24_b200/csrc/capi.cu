@@ -1,0 +1,592 @@
+// capi.cu -- engine (buffer plan, step orchestration, CUDA graph) and the C
+// ABI declared in include/nbody.h.  One time step = Alg. 6:
+//   K1 bbox -> K2 keys -> K3 sort -> K4 permute -> K5 build -> K6 force -> K7 leapfrog
+// all on the context stream, captured once into a CUDA graph and replayed.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "../../include/nbody.h"
+#include "internal.cuh"
+
+using namespace nb;
+
+struct nbody_ctx {
+  int64_t n = 0;
+  double theta = 0.5, eps = 0.0, dt = 0.0;
+  int key_bits_opt = 16;
+  int b = 16;
+  int key_bytes = 8;
+  bool use_graph = true;
+  int traversal = 0;
+  bool timing = false;
+  cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  bool ev_valid = false;
+  int kernels_per_step = 0;
+  int device = 0;
+  int nsm = kNumSMs;
+  cudaStream_t stream = nullptr;
+  cudaStream_t own_stream = nullptr;
+  cudaStream_t cap_stream = nullptr;
+  nbody_status state = NBODY_OK;
+  std::string err;
+  bool loaded = false;
+  bool have_force = false;
+  int64_t steps = 0;
+
+  // device memory arena
+  char* arena = nullptr;
+  float4* pm[2] = {nullptr, nullptr};
+  float4* vi[2] = {nullptr, nullptr};
+  void* keys[2] = {nullptr, nullptr};
+  uint32_t* idx[2] = {nullptr, nullptr};
+  unsigned long long* keys_dbg = nullptr;
+  float4* acc = nullptr;
+  uint32_t* cnt = nullptr;
+  float4* stage = nullptr;
+  float* bbox_part = nullptr;
+  int nbbox = 0;
+  GridInfo* grid = nullptr;
+  unsigned long long* total = nullptr;
+  int* bad = nullptr;
+  SortPlan sort{};
+  TreeView tree{};
+  int perm_buf = 0;
+  bool keys_dbg_valid = false;
+
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+};
+
+namespace {
+
+const char* status_name(nbody_status s) {
+  switch (s) {
+    case NBODY_OK: return "ok";
+    case NBODY_EINVAL: return "invalid argument";
+    case NBODY_ENOMEM: return "out of device memory";
+    case NBODY_ECUDA: return "CUDA error";
+    case NBODY_ENCCL: return "NCCL error";
+    case NBODY_ESTATE: return "bad state";
+  }
+  return "?";
+}
+
+nbody_status fail(nbody_ctx* c, nbody_status s, const std::string& msg) {
+  if (c) {
+    c->err = std::string(status_name(s)) + ": " + msg;
+    if (s == NBODY_ECUDA || s == NBODY_ENCCL) c->state = NBODY_ESTATE;
+  }
+  return s;
+}
+
+#define CK(call)                                                                              \
+  do {                                                                                        \
+    cudaError_t e_ = (call);                                                                  \
+    if (e_ != cudaSuccess) return fail(c, NBODY_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+#define CHECK_CTX(c)                                             \
+  do {                                                           \
+    if (!(c)) return NBODY_EINVAL;                               \
+    if ((c)->state != NBODY_OK) return NBODY_ESTATE;             \
+  } while (0)
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+int resolve_bits(int64_t n, int opt) {
+  if (opt > 0) return opt;
+  int b = 1;
+  while (b < 21 && (uint64_t(1) << (3 * b)) < uint64_t(n)) ++b;  // [A8] smallest b with 8^b >= N
+  return b;
+}
+
+size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
+
+// Tree plan: levels, counts, offsets (sizes follow from N alone).
+int64_t plan_tree(TreeView& t, int64_t n) {
+  t.n = n;
+  t.L = 0;
+  while ((int64_t(1) << t.L) < n) ++t.L;
+  t.count[0] = n;
+  t.off[0] = 0;
+  int64_t total = 0;
+  for (int l = 1; l <= t.L; ++l) {
+    t.count[l] = (t.count[l - 1] + 1) / 2;
+    t.off[l] = total;
+    total += (t.count[l] + 1) & ~int64_t(1);  // keep sibling pairs aligned
+  }
+  for (int l = t.L + 1; l < kMaxLevels; ++l) t.count[l] = t.off[l] = 0;
+  return total;
+}
+
+nbody_status allocate(nbody_ctx* c) {
+  const int64_t n = c->n;
+  const int64_t nodes = plan_tree(c->tree, n);
+  c->nbbox = 2 * c->nsm;
+  const int64_t tiles = sort_tiles(n);
+  size_t sz[32];
+  int k = 0;
+  sz[k++] = 16 * size_t(n);                         // pm0
+  sz[k++] = 16 * size_t(n);                         // pm1
+  sz[k++] = 16 * size_t(n);                         // vi0
+  sz[k++] = 16 * size_t(n);                         // vi1
+  sz[k++] = 8 * size_t(n);                          // keys0
+  sz[k++] = 8 * size_t(n);                          // keys1
+  sz[k++] = 4 * size_t(n);                          // idx0
+  sz[k++] = 4 * size_t(n);                          // idx1
+  sz[k++] = 8 * size_t(n);                          // keys_dbg
+  sz[k++] = 16 * size_t(n);                         // acc
+  sz[k++] = 4 * size_t(n);                          // cnt
+  sz[k++] = 16 * size_t(n);                         // stage
+  sz[k++] = sizeof(float) * 6 * size_t(c->nbbox);   // bbox partials
+  sz[k++] = sizeof(GridInfo);
+  sz[k++] = 8;                                      // total
+  sz[k++] = 8;                                      // bad
+  sz[k++] = sort_scratch_bytes(n);                  // sort
+  sz[k++] = 32 * size_t(nodes);                     // pred
+  sz[k++] = 16 * size_t(nodes);                     // rec
+  sz[k++] = 32 * size_t(nodes);                     // mom
+  sz[k++] = 16 * size_t(nodes);                     // blo
+  sz[k++] = 16 * size_t(nodes);                     // bhi
+  size_t total = 0;
+  for (int i = 0; i < k; ++i) total += align_up(sz[i]);
+  cudaError_t e = cudaMalloc(&c->arena, total);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    c->arena = nullptr;
+    return fail(c, NBODY_ENOMEM, "cudaMalloc of " + std::to_string(total) + " bytes failed");
+  }
+  char* p = c->arena;
+  int i = 0;
+  auto take = [&](void) -> char* { char* r = p; p += align_up(sz[i++]); return r; };
+  c->pm[0] = (float4*)take();
+  c->pm[1] = (float4*)take();
+  c->vi[0] = (float4*)take();
+  c->vi[1] = (float4*)take();
+  c->keys[0] = take();
+  c->keys[1] = take();
+  c->idx[0] = (uint32_t*)take();
+  c->idx[1] = (uint32_t*)take();
+  c->keys_dbg = (unsigned long long*)take();
+  c->acc = (float4*)take();
+  c->cnt = (uint32_t*)take();
+  c->stage = (float4*)take();
+  c->bbox_part = (float*)take();
+  c->grid = (GridInfo*)take();
+  c->total = (unsigned long long*)take();
+  c->bad = (int*)take();
+  char* sortmem = take();
+  c->tree.pred = (double4*)take();
+  c->tree.rec = (float4*)take();
+  c->tree.mom = (double4*)take();
+  c->tree.blo = (float4*)take();
+  c->tree.bhi = (float4*)take();
+  c->sort.n = n;
+  c->sort.tiles = tiles;
+  c->sort.ghist = (uint32_t*)sortmem;
+  c->sort.tile_ctr = c->sort.ghist + 8 * 256;
+  c->sort.status = c->sort.tile_ctr + 8;
+  return NBODY_OK;
+}
+
+void drop_graph(nbody_ctx* c) {
+  if (c->gexec) cudaGraphExecDestroy(c->gexec);
+  if (c->graph) cudaGraphDestroy(c->graph);
+  c->gexec = nullptr;
+  c->graph = nullptr;
+}
+
+// One force pass (and optionally the update) on stream s.  State enters in
+// (pm[0], vi[0]) in the current slot order and leaves there in the new
+// Hilbert order.
+nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool debug) {
+  const int64_t n = c->n;
+  const bool tm = c->timing && s == c->stream;
+  auto mark = [&](int i) -> cudaError_t { return tm ? cudaEventRecord(c->ev[i], s) : cudaSuccess; };
+  CK(mark(0));
+  launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
+  launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
+  if (c->key_bytes == 4)
+    launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), s);
+  else
+    launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), s);
+  if (debug) {
+    CK(cudaMemcpyAsync(c->keys_dbg, c->keys[0], size_t(c->key_bytes) * n, cudaMemcpyDeviceToDevice, s));
+  }
+  CK(mark(1));
+  c->perm_buf = launch_radix_sort(c->sort, c->keys, c->idx, s);
+  CK(mark(2));
+  launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
+  launch_build(c->tree, c->pm[1], s);
+  CK(cudaMemsetAsync(c->total, 0, sizeof(unsigned long long), s));
+  CK(mark(3));
+  ForceParams fp;
+  fp.t = c->tree;
+  fp.leaves = c->pm[1];
+  fp.t_begin = 0;
+  fp.t_end = n;
+  fp.th2 = c->theta * c->theta;
+  fp.eps2 = float(c->eps * c->eps);
+  fp.acc = c->acc;
+  fp.count = c->cnt;
+  fp.total = c->total;
+  launch_force(fp, c->traversal, s);
+  CK(mark(4));
+  if (integrate) {
+    launch_leapfrog(c->pm[1], c->vi[1], c->acc, n, float(c->dt), c->pm[0], c->vi[0], s);
+  } else {
+    CK(cudaMemcpyAsync(c->pm[0], c->pm[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(c->vi[0], c->vi[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+  }
+  CK(mark(5));
+  c->ev_valid = tm;
+  // K1 2 + K2 1 + K3 (1 + passes) + K4 1 + K5 L + K6 1 + K7 1
+  c->kernels_per_step = 2 + 1 + 1 + c->sort.passes + 1 + c->tree.L + 1 + (integrate ? 1 : 0);
+  CK(cudaGetLastError());
+  return NBODY_OK;
+}
+
+nbody_status build_graph(nbody_ctx* c) {
+  drop_graph(c);
+  CK(cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal));
+  nbody_status st = enqueue_pass(c, c->cap_stream, true, false);
+  cudaGraph_t g = nullptr;
+  cudaError_t e = cudaStreamEndCapture(c->cap_stream, &g);
+  if (st != NBODY_OK) {
+    if (g) cudaGraphDestroy(g);
+    return st;
+  }
+  if (e != cudaSuccess) return fail(c, NBODY_ECUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+  c->graph = g;
+  CK(cudaGraphInstantiate(&c->gexec, g, 0));
+  return NBODY_OK;
+}
+
+nbody_status sync_stream(nbody_ctx* c) {
+  CK(cudaStreamSynchronize(c->stream));
+  return NBODY_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int nbody_version(void) { return 100; }
+
+nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx** out) {
+  if (!out) return NBODY_EINVAL;
+  *out = nullptr;
+  if (n < 1 || n >= (int64_t(1) << 30)) return NBODY_EINVAL;
+  if (!std::isfinite(theta) || theta < 0 || !std::isfinite(eps) || eps < 0 || !std::isfinite(dt)) return NBODY_EINVAL;
+  nbody_ctx* c = new (std::nothrow) nbody_ctx;
+  if (!c) return NBODY_ENOMEM;
+  c->n = n;
+  c->theta = theta;
+  c->eps = eps;
+  c->dt = dt;
+  auto bail = [&](nbody_status s) {
+    nbody_destroy(c);
+    return s;
+  };
+  if (cudaGetDevice(&c->device) != cudaSuccess) return bail(NBODY_ECUDA);
+  cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device);
+  if (c->nsm <= 0) c->nsm = kNumSMs;
+  if (cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking) != cudaSuccess) return bail(NBODY_ECUDA);
+  if (cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking) != cudaSuccess) return bail(NBODY_ECUDA);
+  for (auto& e : c->ev)
+    if (cudaEventCreate(&e) != cudaSuccess) return bail(NBODY_ECUDA);
+  c->stream = c->own_stream;
+  nbody_status s = allocate(c);
+  if (s != NBODY_OK) return bail(s);
+  c->b = resolve_bits(n, c->key_bits_opt);
+  c->key_bytes = 3 * c->b <= 32 ? 4 : 8;
+  c->sort.key_bytes = c->key_bytes;
+  c->sort.passes = (3 * c->b + 7) / 8;
+  *out = c;
+  return NBODY_OK;
+}
+
+nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
+  CHECK_CTX(c);
+  switch (option) {
+    case NBODY_OPT_KEY_BITS:
+      if (value < 0 || value > 21) return fail(c, NBODY_EINVAL, "key bits must be in [0, 21]");
+      c->key_bits_opt = int(value);
+      c->b = resolve_bits(c->n, c->key_bits_opt);
+      c->key_bytes = 3 * c->b <= 32 ? 4 : 8;
+      c->sort.key_bytes = c->key_bytes;
+      c->sort.passes = (3 * c->b + 7) / 8;
+      drop_graph(c);
+      return NBODY_OK;
+    case NBODY_OPT_STREAM:
+      c->stream = value ? reinterpret_cast<cudaStream_t>(value) : c->own_stream;
+      return NBODY_OK;
+    case NBODY_OPT_USE_GRAPH:
+      if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "use_graph must be 0 or 1");
+      c->use_graph = value != 0;
+      return NBODY_OK;
+    case NBODY_OPT_TIMING:
+      if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "timing must be 0 or 1");
+      c->timing = value != 0;
+      return NBODY_OK;
+    case NBODY_OPT_TRAVERSAL:
+      if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown traversal variant");
+      c->traversal = int(value);
+      drop_graph(c);
+      return NBODY_OK;
+    default:
+      return fail(c, NBODY_EINVAL, "unknown option " + std::to_string(option));
+  }
+}
+
+nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, const float* mass) {
+  CHECK_CTX(c);
+  if (!pos || !vel || !mass) return fail(c, NBODY_EINVAL, "null input");
+  const int64_t n = c->n;
+  const float *dp = pos, *dv = vel, *dm = mass;
+  cudaStream_t s = c->stream;
+  if (!is_device_ptr(pos)) {
+    CK(cudaMemcpyAsync(c->acc, pos, 12 * size_t(n), cudaMemcpyDefault, s));
+    dp = reinterpret_cast<const float*>(c->acc);
+  }
+  if (!is_device_ptr(vel)) {
+    CK(cudaMemcpyAsync(c->stage, vel, 12 * size_t(n), cudaMemcpyDefault, s));
+    dv = reinterpret_cast<const float*>(c->stage);
+  }
+  if (!is_device_ptr(mass)) {
+    CK(cudaMemcpyAsync(c->cnt, mass, 4 * size_t(n), cudaMemcpyDefault, s));
+    dm = reinterpret_cast<const float*>(c->cnt);
+  }
+  CK(cudaMemsetAsync(c->bad, 0, sizeof(int), s));
+  launch_pack_bodies(dp, dv, dm, n, c->pm[0], c->vi[0], c->bad, s);
+  CK(cudaGetLastError());
+  int bad = 0;
+  CK(cudaMemcpyAsync(&bad, c->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (bad) {
+    c->loaded = false;
+    return fail(c, NBODY_EINVAL, (bad & 2) ? "masses must be finite and > 0" : "non-finite position or velocity");
+  }
+  c->loaded = true;
+  c->have_force = false;
+  c->keys_dbg_valid = false;
+  c->steps = 0;
+  return NBODY_OK;
+}
+
+nbody_status nbody_compute_accel(nbody_ctx* c) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  nbody_status s = enqueue_pass(c, c->stream, false, true);
+  if (s != NBODY_OK) return s;
+  c->have_force = true;
+  c->keys_dbg_valid = true;
+  c->steps += 0;
+  return NBODY_OK;
+}
+
+nbody_status nbody_step(nbody_ctx* c, int nsteps) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (nsteps < 0) return fail(c, NBODY_EINVAL, "nsteps < 0");
+  if (nsteps == 0) return NBODY_OK;
+  if (c->use_graph) {
+    if (!c->gexec) {
+      nbody_status s = build_graph(c);
+      if (s != NBODY_OK) return s;
+    }
+    for (int i = 0; i < nsteps; ++i) CK(cudaGraphLaunch(c->gexec, c->stream));
+    c->ev_valid = false;
+  } else {
+    for (int i = 0; i < nsteps; ++i) {
+      nbody_status s = enqueue_pass(c, c->stream, true, false);
+      if (s != NBODY_OK) return s;
+    }
+  }
+  c->have_force = true;
+  c->keys_dbg_valid = false;
+  c->steps += nsteps;
+  return NBODY_OK;
+}
+
+nbody_status nbody_sync(nbody_ctx* c) {
+  CHECK_CTX(c);
+  return sync_stream(c);
+}
+
+static nbody_status get_by_id3(nbody_ctx* c, const float4* src, float* out) {
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  const int64_t n = c->n;
+  if (is_device_ptr(out)) {
+    launch_scatter_by_id3(src, c->vi[0], n, out, c->stream);
+    CK(cudaGetLastError());
+    return sync_stream(c);
+  }
+  float* tmp = reinterpret_cast<float*>(c->stage);
+  launch_scatter_by_id3(src, c->vi[0], n, tmp, c->stream);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(out, tmp, 12 * size_t(n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
+nbody_status nbody_get_accel(nbody_ctx* c, float* out) {
+  CHECK_CTX(c);
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  return get_by_id3(c, c->acc, out);
+}
+
+nbody_status nbody_get_positions(nbody_ctx* c, float* out) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  return get_by_id3(c, c->pm[0], out);
+}
+
+nbody_status nbody_get_velocities(nbody_ctx* c, float* out) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  return get_by_id3(c, c->vi[0], out);
+}
+
+nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
+  CHECK_CTX(c);
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  const int64_t n = c->n;
+  if (is_device_ptr(out)) {
+    launch_scatter_by_id1(c->cnt, c->vi[0], n, out, c->stream);
+    CK(cudaGetLastError());
+    return sync_stream(c);
+  }
+  uint32_t* tmp = reinterpret_cast<uint32_t*>(c->stage);
+  launch_scatter_by_id1(c->cnt, c->vi[0], n, tmp, c->stream);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(out, tmp, 4 * size_t(n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
+nbody_status nbody_get_state(nbody_ctx* c, float* pos_m, float* vel_id) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (pos_m) CK(cudaMemcpyAsync(pos_m, c->pm[0], 16 * size_t(c->n), cudaMemcpyDefault, c->stream));
+  if (vel_id) CK(cudaMemcpyAsync(vel_id, c->vi[0], 16 * size_t(c->n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
+nbody_status nbody_get_stats(nbody_ctx* c, nbody_stats* out) {
+  CHECK_CTX(c);
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  std::memset(out, 0, sizeof(*out));
+  out->n = c->n;
+  out->key_bits = c->b;
+  out->levels = c->tree.L;
+  out->steps = c->steps;
+  if (c->have_force) {
+    unsigned long long t = 0;
+    CK(cudaMemcpyAsync(&t, c->total, sizeof(t), cudaMemcpyDeviceToHost, c->stream));
+    nbody_status s = sync_stream(c);
+    if (s != NBODY_OK) return s;
+    out->interactions = t;
+  }
+  out->kernels_per_step = c->kernels_per_step;
+  if (c->ev_valid) {
+    CK(cudaEventSynchronize(c->ev[5]));
+    float* dst[5] = {&out->ms_bbox_keys, &out->ms_sort, &out->ms_build, &out->ms_force, &out->ms_update};
+    for (int i = 0; i < 5; ++i) CK(cudaEventElapsedTime(dst[i], c->ev[i], c->ev[i + 1]));
+  }
+  return NBODY_OK;
+}
+
+nbody_status nbody_debug_keys(nbody_ctx* c, uint64_t* keys) {
+  CHECK_CTX(c);
+  if (!keys) return fail(c, NBODY_EINVAL, "null output");
+  if (!c->keys_dbg_valid) return fail(c, NBODY_ESTATE, "keys are kept by nbody_compute_accel only");
+  const int64_t n = c->n;
+  if (c->key_bytes == 8) {
+    CK(cudaMemcpyAsync(keys, c->keys_dbg, 8 * size_t(n), cudaMemcpyDefault, c->stream));
+    return sync_stream(c);
+  }
+  // widen u32 keys on the host side of the copy
+  uint32_t* tmp = new (std::nothrow) uint32_t[size_t(n)];
+  if (!tmp) return fail(c, NBODY_ENOMEM, "host buffer");
+  cudaError_t e = cudaMemcpyAsync(tmp, c->keys_dbg, 4 * size_t(n), cudaMemcpyDefault, c->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+  if (e != cudaSuccess) {
+    delete[] tmp;
+    return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
+  }
+  const bool dev = is_device_ptr(keys);
+  if (!dev) {
+    for (int64_t i = 0; i < n; ++i) keys[i] = tmp[i];
+    delete[] tmp;
+    return NBODY_OK;
+  }
+  uint64_t* wide = new (std::nothrow) uint64_t[size_t(n)];
+  if (!wide) {
+    delete[] tmp;
+    return fail(c, NBODY_ENOMEM, "host buffer");
+  }
+  for (int64_t i = 0; i < n; ++i) wide[i] = tmp[i];
+  e = cudaMemcpy(keys, wide, 8 * size_t(n), cudaMemcpyDefault);
+  delete[] tmp;
+  delete[] wide;
+  if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
+  return NBODY_OK;
+}
+
+nbody_status nbody_debug_perm(nbody_ctx* c, uint32_t* perm) {
+  CHECK_CTX(c);
+  if (!perm) return fail(c, NBODY_EINVAL, "null output");
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  CK(cudaMemcpyAsync(perm, c->idx[c->perm_buf], 4 * size_t(c->n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
+nbody_status nbody_debug_level(nbody_ctx* c, int level, int64_t* count, double* pred, float* rec, float* box) {
+  CHECK_CTX(c);
+  if (level < 1 || level > c->tree.L) return fail(c, NBODY_EINVAL, "level out of range [1, L]");
+  const int64_t cnt = c->tree.count[level];
+  if (count) *count = cnt;
+  if (!pred && !rec && !box) return NBODY_OK;
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  const int64_t off = c->tree.off[level];
+  cudaStream_t s = c->stream;
+  if (pred) CK(cudaMemcpyAsync(pred, c->tree.pred + off, 32 * size_t(cnt), cudaMemcpyDefault, s));
+  if (rec) CK(cudaMemcpyAsync(rec, c->tree.rec + off, 16 * size_t(cnt), cudaMemcpyDefault, s));
+  if (box) {
+    CK(cudaMemcpy2DAsync(box, 24, c->tree.blo + off, 16, 12, size_t(cnt), cudaMemcpyDefault, s));
+    CK(cudaMemcpy2DAsync(box + 3, 24, c->tree.bhi + off, 16, 12, size_t(cnt), cudaMemcpyDefault, s));
+  }
+  return sync_stream(c);
+}
+
+const char* nbody_last_error(const nbody_ctx* c) {
+  if (!c) return "null context";
+  return c->err.c_str();
+}
+
+void nbody_destroy(nbody_ctx* c) {
+  if (!c) return;
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  drop_graph(c);
+  if (c->arena) cudaFree(c->arena);
+  for (auto& e : c->ev)
+    if (e) cudaEventDestroy(e);
+  if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
+  if (c->own_stream) cudaStreamDestroy(c->own_stream);
+  cudaGetLastError();
+  delete c;
+}
+
+}  // extern "C"

@@ -1,0 +1,92 @@
+// internal.cuh -- device data layout and kernel launchers of the B200 path.
+//
+// Product code only: nothing here is shared with oracle/ (DESIGN.md
+// "Independence").  P:NNN = line of the paper text; [A#] = DESIGN.md reading.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace nb {
+
+constexpr int kMaxLevels = 32;   // L = ceil(log2 N) <= 30 for N < 2^30
+constexpr int kNumSMs = 148;     // B200; the engine re-reads the device's count
+
+// Grid of the Hilbert quantisation computed on the device each step
+// from the bounding box (Alg. 3).
+struct GridInfo {
+  float lo[3];
+  float hi[3];
+  double inv;    // 2^b / ext, or 0 when ext == 0 [A17]
+  int b;         // bits per axis
+  int pad;
+};
+
+// Balanced, ragged BVH stored level by level ([A6]).  Level 0 is the
+// sorted body array itself; internal node (l, j), l >= 1, lives at
+// off[l] + j of each per-node array (off[l] even, so sibling pairs are
+// 2-node aligned).
+struct TreeView {
+  int L;                       // levels above the leaves
+  int64_t n;                   // bodies (= nodes at level 0)
+  int64_t count[kMaxLevels];   // nodes per level: ceil(n / 2^l)
+  int64_t off[kMaxLevels];     // start of level l in the node arrays
+  double4* pred;   // (com64 x, y, z, s^2)   opening test data, fp64 [A3][A16]
+  float4* rec;     // ((float)com64, (float)M) monopole for the interaction
+  double4* mom;    // (M, Mx, My, Mz) fp64 moments (build only) [A12]
+  float4* blo;     // AABB lo (x, y, z, -)
+  float4* bhi;     // AABB hi (x, y, z, -)
+};
+
+struct ForceParams {
+  TreeView t;
+  const float4* leaves;   // sorted (x, y, z, m)
+  int64_t t_begin;        // owned target slots [t_begin, t_end)
+  int64_t t_end;
+  double th2;             // theta^2 (fp64, used by the opening test)
+  float eps2;             // eps^2 (fp32 interaction)
+  float4* acc;            // per owned slot (ax, ay, az, 0), indexed slot - t_begin
+  uint32_t* count;        // interactions per owned slot
+  unsigned long long* total;  // sum of interactions (integer atomics only)
+};
+
+// ---- K1 / K2 --------------------------------------------------------------
+void launch_bbox_partial(const float4* pm, int64_t n, float* partial, int nblocks, cudaStream_t s);
+void launch_bbox_final(const float* partial, int nparts, int b, GridInfo* g, cudaStream_t s);
+void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, cudaStream_t s);
+void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, cudaStream_t s);
+
+// ---- K3 radix sort ---------------------------------------------------------
+struct SortPlan {
+  int64_t n;
+  int key_bytes;      // 4 or 8
+  int passes;         // ceil(3b / 8)
+  int64_t tiles;      // per pass
+  uint32_t* ghist;    // [8][256]
+  uint32_t* status;   // [passes][tiles][256]
+  uint32_t* tile_ctr; // [8]
+};
+int64_t sort_tiles(int64_t n);
+size_t sort_scratch_bytes(int64_t n);
+// Sorts (keys[0], implicit iota) into perm; keys/idx double buffers are
+// clobbered.  Returns the buffer index (0/1) of idx holding the permutation.
+int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s);
+
+// ---- K4 / K5 ---------------------------------------------------------------
+void launch_permute(const float4* pm_in, const float4* vi_in, const uint32_t* perm, int64_t n, float4* pm_out,
+                    float4* vi_out, cudaStream_t s);
+void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);
+
+// ---- K6 --------------------------------------------------------------------
+void launch_force(const ForceParams& p, int variant, cudaStream_t s);
+
+// ---- K7 and helpers --------------------------------------------------------
+void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
+                     float4* vi_out, cudaStream_t s);
+void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
+                        int* bad, cudaStream_t s);
+// out[id][3] <- src[slot].xyz for slots [0, n); id from vi[slot].w
+void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s);
+void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s);
+
+}  // namespace nb

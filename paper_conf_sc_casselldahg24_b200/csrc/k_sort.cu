@@ -1,0 +1,248 @@
+// K3 HILBERTSORT (Alg. 7): stable LSD radix sort of (key, slot)
+// pairs, applied afterwards as a permutation.  [A10] stability makes
+// ties keep the current slot order, the same result as std::stable_sort.
+//
+// Onesweep structure (one upfront histogram pass over all digits, then one
+// kernel per 8-bit digit):
+//   * tiles of 512 threads x 8 keys = 4096 keys, tile ids from an atomic
+//     counter so every tile only ever waits on tiles that already run;
+//   * ranking inside a warp with __match_any_sync (warp multisplit), across
+//     the 16 warps of a tile by per-warp shared-memory histograms;
+//   * decoupled look-back over per-(tile, digit) status words (2 flag bits +
+//     30 count bits, so N < 2^30);
+//   * scatter through shared memory in digit order so that the global stores
+//     of a tile are runs of consecutive addresses.
+// HBM bound: per pass 2 x (key + 4 B) per body; the upfront histogram reads
+// the keys once.
+#include <cuda/atomic>
+
+#include "internal.cuh"
+
+namespace nb {
+namespace {
+
+constexpr int kThreads = 512;
+constexpr int kWarps = kThreads / 32;
+constexpr int kItems = 8;
+constexpr int kTile = kThreads * kItems;
+constexpr int kRadix = 256;
+constexpr uint32_t kFlagAgg = 1u << 30;
+constexpr uint32_t kFlagInc = 1u << 31;
+constexpr uint32_t kValMask = kFlagAgg - 1u;
+
+template <class K>
+__device__ __forceinline__ uint32_t digit_of(K k, int shift) {
+  return uint32_t(k >> shift) & (kRadix - 1);
+}
+
+// Histograms of every digit position in one read of the keys; warp-aggregated
+// shared-memory counts (Hilbert keys are heavily skewed in the high digits).
+template <class K>
+__global__ __launch_bounds__(kThreads) void k_hist(const K* __restrict__ keys, int64_t n, int passes,
+                                                   uint32_t* __restrict__ ghist) {
+  __shared__ uint32_t sh[8 * kRadix];
+  for (int i = threadIdx.x; i < passes * kRadix; i += kThreads) sh[i] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = int64_t(gridDim.x) * kThreads;
+  for (int64_t base = int64_t(blockIdx.x) * kThreads + (threadIdx.x & ~31); base < n; base += stride) {
+    const int64_t i = base + lane;
+    const bool ok = i < n;
+    const K k = ok ? keys[i] : K(0);
+    for (int p = 0; p < passes; ++p) {
+      const uint32_t d = ok ? digit_of(k, 8 * p) : kRadix;
+      const uint32_t peers = __match_any_sync(0xffffffffu, d);
+      if (ok && lane == __ffs(peers) - 1) atomicAdd(&sh[p * kRadix + d], uint32_t(__popc(peers)));
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < passes * kRadix; i += kThreads)
+    if (sh[i]) atomicAdd(&ghist[i], sh[i]);
+}
+
+// Exclusive scan of v over threads 0..255 (others pass 0); every thread of
+// the block must call.  Returns the exclusive prefix for the caller.
+__device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t* s_tmp) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31 && w < kRadix / 32) s_tmp[w] = x;
+  __syncthreads();
+  uint32_t pre = 0;
+  if (w < kRadix / 32)
+    for (int j = 0; j < w; ++j) pre += s_tmp[j];
+  __syncthreads();
+  return pre + x - v;
+}
+
+template <class K, bool kFirst, bool kWriteKeys>
+__global__ __launch_bounds__(kThreads) void k_onesweep(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                       K* __restrict__ kout, uint32_t* __restrict__ vout, int64_t n,
+                                                       int shift, const uint32_t* __restrict__ ghist,
+                                                       uint32_t* __restrict__ status, uint32_t* __restrict__ tile_ctr) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  uint32_t* s_whist = reinterpret_cast<uint32_t*>(smem);                  // [kWarps][256]
+  K* s_keys = reinterpret_cast<K*>(s_whist + kWarps * kRadix);            // [kTile]
+  uint32_t* s_vals = reinterpret_cast<uint32_t*>(s_keys + kTile);         // [kTile]
+  __shared__ uint32_t s_dlocal[kRadix], s_dglobal[kRadix], s_tmp[kWarps];
+  __shared__ uint32_t s_tile;
+
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  for (int i = tid; i < kWarps * kRadix; i += kThreads) s_whist[i] = 0;
+  __syncthreads();
+  const int64_t tile = s_tile;
+  const int64_t base = tile * kTile;
+
+  K k[kItems];
+  uint32_t v[kItems], d[kItems], r[kItems];
+#pragma unroll
+  for (int i = 0; i < kItems; ++i) {
+    const int64_t pos = base + w * (32 * kItems) + i * 32 + lane;
+    const bool ok = pos < n;
+    k[i] = ok ? kin[pos] : K(0);
+    v[i] = kFirst ? uint32_t(pos) : (ok ? vin[pos] : 0u);
+    d[i] = ok ? digit_of(k[i], shift) : uint32_t(kRadix);
+  }
+  // Rank inside the warp, in (item, lane) order = position order: stable.
+  uint32_t* wh = s_whist + w * kRadix;
+#pragma unroll
+  for (int i = 0; i < kItems; ++i) {
+    const uint32_t peers = __match_any_sync(0xffffffffu, d[i]);
+    const int leader = __ffs(peers) - 1;
+    const uint32_t below = __popc(peers & ((1u << lane) - 1u));
+    uint32_t pre = 0;
+    if (lane == leader && d[i] < kRadix) {
+      pre = wh[d[i]];
+      wh[d[i]] = pre + __popc(peers);
+    }
+    pre = __shfl_sync(0xffffffffu, pre, leader);
+    r[i] = pre + below;
+    __syncwarp();
+  }
+  __syncthreads();
+
+  // Per digit: exclusive prefix over warps (in place) and the tile count.
+  uint32_t cnt = 0;
+  if (tid < kRadix) {
+    for (int j = 0; j < kWarps; ++j) {
+      const uint32_t c = s_whist[j * kRadix + tid];
+      s_whist[j * kRadix + tid] = cnt;
+      cnt += c;
+    }
+  }
+  const uint32_t dl = scan256(tid < kRadix ? cnt : 0u, s_tmp);
+  const uint32_t gb = scan256(tid < kRadix ? ghist[tid] : 0u, s_tmp);
+  if (tid < kRadix) {
+    s_dlocal[tid] = dl;
+    cuda::atomic_ref<uint32_t, cuda::thread_scope_device> mine(status[tile * kRadix + tid]);
+    if (tile == 0) {
+      mine.store(kFlagInc | cnt, cuda::memory_order_relaxed);
+      s_dglobal[tid] = gb;
+    } else {
+      mine.store(kFlagAgg | cnt, cuda::memory_order_relaxed);
+      uint32_t excl = 0;
+      int64_t p = tile - 1;
+      for (;;) {
+        cuda::atomic_ref<uint32_t, cuda::thread_scope_device> o(status[p * kRadix + tid]);
+        const uint32_t s = o.load(cuda::memory_order_relaxed);
+        if ((s & ~kValMask) == 0) continue;  // predecessor not published yet
+        excl += s & kValMask;
+        if (s & kFlagInc) break;
+        --p;
+      }
+      mine.store(kFlagInc | (excl + cnt), cuda::memory_order_relaxed);
+      s_dglobal[tid] = gb + excl;
+    }
+  }
+  __syncthreads();
+
+  // Scatter into shared memory in digit order ...
+#pragma unroll
+  for (int i = 0; i < kItems; ++i) {
+    if (d[i] < kRadix) {
+      const uint32_t pos = s_dlocal[d[i]] + s_whist[w * kRadix + d[i]] + r[i];
+      s_keys[pos] = k[i];
+      s_vals[pos] = v[i];
+    }
+  }
+  __syncthreads();
+  // ... and write runs of consecutive global addresses.
+  const int valid = int(n - base < kTile ? n - base : int64_t(kTile));
+  for (int j = tid; j < valid; j += kThreads) {
+    const K key = s_keys[j];
+    const uint32_t dd = digit_of(key, shift);
+    const int64_t g = int64_t(s_dglobal[dd]) + (j - int64_t(s_dlocal[dd]));
+    if (kWriteKeys) kout[g] = key;
+    vout[g] = s_vals[j];
+  }
+}
+
+template <class K>
+constexpr size_t dyn_smem() {
+  return sizeof(uint32_t) * kWarps * kRadix + sizeof(K) * kTile + sizeof(uint32_t) * kTile;
+}
+
+template <class K, bool F, bool W>
+void set_attr() {
+  cudaFuncSetAttribute(k_onesweep<K, F, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn_smem<K>()));
+}
+
+template <class K>
+void run_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s) {
+  static bool attrs = false;
+  if (!attrs) {
+    set_attr<K, true, true>(); set_attr<K, true, false>();
+    set_attr<K, false, true>(); set_attr<K, false, false>();
+    attrs = true;
+  }
+  cudaMemsetAsync(p.ghist, 0, sizeof(uint32_t) * 8 * kRadix, s);
+  cudaMemsetAsync(p.tile_ctr, 0, sizeof(uint32_t) * 8, s);
+  cudaMemsetAsync(p.status, 0, sizeof(uint32_t) * size_t(p.passes) * size_t(p.tiles) * kRadix, s);
+  const int hb = int(p.tiles < 4 * kNumSMs ? p.tiles : int64_t(4 * kNumSMs));
+  k_hist<K><<<hb, kThreads, 0, s>>>(static_cast<const K*>(keys[0]), p.n, p.passes, p.ghist);
+  for (int pass = 0; pass < p.passes; ++pass) {
+    const int in = pass & 1, out = in ^ 1;
+    const K* kin = static_cast<const K*>(keys[in]);
+    K* kout = static_cast<K*>(keys[out]);
+    const bool first = pass == 0, last = pass == p.passes - 1;
+    uint32_t* st = p.status + size_t(pass) * size_t(p.tiles) * kRadix;
+    const uint32_t* gh = p.ghist + pass * kRadix;
+    const unsigned grid = unsigned(p.tiles);
+    const size_t sm = dyn_smem<K>();
+    if (first && last)
+      k_onesweep<K, true, false><<<grid, kThreads, sm, s>>>(kin, idx[in], kout, idx[out], p.n, 8 * pass, gh, st,
+                                                          p.tile_ctr + pass);
+    else if (first)
+      k_onesweep<K, true, true><<<grid, kThreads, sm, s>>>(kin, idx[in], kout, idx[out], p.n, 8 * pass, gh, st,
+                                                         p.tile_ctr + pass);
+    else if (last)
+      k_onesweep<K, false, false><<<grid, kThreads, sm, s>>>(kin, idx[in], kout, idx[out], p.n, 8 * pass, gh, st,
+                                                           p.tile_ctr + pass);
+    else
+      k_onesweep<K, false, true><<<grid, kThreads, sm, s>>>(kin, idx[in], kout, idx[out], p.n, 8 * pass, gh, st,
+                                                          p.tile_ctr + pass);
+  }
+}
+
+}  // namespace
+
+int64_t sort_tiles(int64_t n) { return (n + kTile - 1) / kTile; }
+
+size_t sort_scratch_bytes(int64_t n) {
+  return sizeof(uint32_t) * (8 * kRadix + 8 + size_t(8) * size_t(sort_tiles(n)) * kRadix);
+}
+
+int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s) {
+  if (p.key_bytes == 4)
+    run_sort<uint32_t>(p, keys, idx, s);
+  else
+    run_sort<unsigned long long>(p, keys, idx, s);
+  return p.passes & 1;
+}
+
+}  // namespace nb

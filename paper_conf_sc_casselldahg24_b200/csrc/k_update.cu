@@ -1,0 +1,85 @@
+// K7 UPDATEPOSITION (Stormer-Verlet; ref [12]) as kick-drift
+// leapfrog on half-step velocities [A14]: v_{+1/2} = v_{-1/2} + a dt,
+// x_{t+1} = x_t + v_{+1/2} dt (fp32 FMA).  Plus the body packing / id
+// scatter helpers of the C ABI.  All HBM bound, one thread per body.
+#include "internal.cuh"
+
+namespace nb {
+namespace {
+
+__global__ __launch_bounds__(256) void k_leapfrog(const float4* __restrict__ pm_in, const float4* __restrict__ vi_in,
+                                                  const float4* __restrict__ acc, int64_t n, float dt,
+                                                  float4* __restrict__ pm_out, float4* __restrict__ vi_out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  float4 p = pm_in[i], v = vi_in[i];
+  const float4 a = acc[i];
+  v.x = fmaf(a.x, dt, v.x);
+  v.y = fmaf(a.y, dt, v.y);
+  v.z = fmaf(a.z, dt, v.z);
+  p.x = fmaf(v.x, dt, p.x);
+  p.y = fmaf(v.y, dt, p.y);
+  p.z = fmaf(v.z, dt, p.z);
+  pm_out[i] = p;
+  vi_out[i] = v;
+}
+
+// pos[n][3], vel[n][3], mass[n] -> (x, y, z, m), (vx, vy, vz, id bits).
+// *bad |= 1 for a non-finite position/velocity, 2 for a mass <= 0 or
+// non-finite [A18].
+__global__ __launch_bounds__(256) void k_pack(const float* __restrict__ pos, const float* __restrict__ vel,
+                                              const float* __restrict__ mass, int64_t n, float4* __restrict__ pm,
+                                              float4* __restrict__ vi, int* __restrict__ bad) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const float x = pos[3 * i], y = pos[3 * i + 1], z = pos[3 * i + 2];
+  const float u = vel[3 * i], v = vel[3 * i + 1], w = vel[3 * i + 2];
+  const float m = mass[i];
+  int flag = 0;
+  if (!(isfinite(x) && isfinite(y) && isfinite(z) && isfinite(u) && isfinite(v) && isfinite(w))) flag |= 1;
+  if (!(isfinite(m) && m > 0.f)) flag |= 2;
+  if (flag) atomicOr(bad, flag);
+  pm[i] = make_float4(x, y, z, m);
+  vi[i] = make_float4(u, v, w, __int_as_float(int(i)));
+}
+
+__global__ __launch_bounds__(256) void k_scatter3(const float4* __restrict__ src, const float4* __restrict__ vi,
+                                                  int64_t n, float* __restrict__ out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int64_t id = __float_as_int(vi[i].w);
+  const float4 s = src[i];
+  out[3 * id] = s.x;
+  out[3 * id + 1] = s.y;
+  out[3 * id + 2] = s.z;
+}
+
+__global__ __launch_bounds__(256) void k_scatter1(const uint32_t* __restrict__ src, const float4* __restrict__ vi,
+                                                  int64_t n, uint32_t* __restrict__ out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  out[__float_as_int(vi[i].w)] = src[i];
+}
+
+}  // namespace
+
+void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
+                     float4* vi_out, cudaStream_t s) {
+  if (n <= 0) return;
+  k_leapfrog<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, n, dt, pm_out, vi_out);
+}
+
+void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
+                        int* bad, cudaStream_t s) {
+  k_pack<<<unsigned((n + 255) / 256), 256, 0, s>>>(pos, vel, mass, n, pm, vi, bad);
+}
+
+void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s) {
+  k_scatter3<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
+}
+
+void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s) {
+  k_scatter1<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
+}
+
+}  // namespace nb

@@ -1,0 +1,150 @@
+"""Thin Python wrapper over the C ABI (include/nbody.h).
+
+Arrays may be numpy arrays (host) or torch tensors (host or CUDA); they are
+passed to the library by pointer.  PyTorch supplies device memory, streams
+and process groups only -- every stage of the step runs in libnbody_b200.so.
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from . import _capi
+
+
+def _ptr(a) -> int:
+    """Raw pointer of a C-contiguous numpy array or torch tensor."""
+    if isinstance(a, np.ndarray):
+        if not a.flags["C_CONTIGUOUS"]:
+            raise ValueError("array must be C-contiguous")
+        return a.ctypes.data
+    if hasattr(a, "data_ptr"):
+        if not a.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        return a.data_ptr()
+    if isinstance(a, int):
+        return a
+    raise TypeError(f"unsupported buffer type {type(a)}")
+
+
+def _f32(a, n, cols):
+    if isinstance(a, np.ndarray):
+        a = np.ascontiguousarray(a, dtype=np.float32)
+        if a.size != n * cols:
+            raise ValueError(f"expected {n}x{cols} values, got {a.shape}")
+        return a
+    if hasattr(a, "data_ptr"):
+        import torch
+        if a.dtype != torch.float32 or a.numel() != n * cols:
+            raise ValueError("expected a float32 tensor of n*cols elements")
+        return a.contiguous()
+    raise TypeError(type(a))
+
+
+class NBody:
+    """One simulation context: ``NBody(n, theta, eps, dt)``."""
+
+    def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
+                 stream=None, use_graph: bool = True, traversal: int = 0):
+        self.lib = _capi.load()
+        self.n = int(n)
+        h = C.c_void_p()
+        st = self.lib.nbody_create(self.n, float(theta), float(eps), float(dt), C.byref(h))
+        if st != 0:
+            raise _capi.NBodyError(st, "nbody_create failed")
+        self.h = h
+        self.set_option(_capi.NBODY_OPT_KEY_BITS, key_bits)
+        self.set_option(_capi.NBODY_OPT_USE_GRAPH, int(use_graph))
+        self.set_option(_capi.NBODY_OPT_TRAVERSAL, traversal)
+        if stream is not None:
+            self.set_option(_capi.NBODY_OPT_STREAM, int(stream))
+
+    # -- lifecycle ---------------------------------------------------------
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.nbody_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def _ck(self, st):
+        _capi.check(self.h, st)
+
+    # -- calls -------------------------------------------------------------
+    def set_option(self, opt: int, value: int):
+        self._ck(self.lib.nbody_set_option(self.h, int(opt), int(value)))
+
+    def set_bodies(self, pos, vel, mass):
+        p, v, m = _f32(pos, self.n, 3), _f32(vel, self.n, 3), _f32(mass, self.n, 1)
+        self._ck(self.lib.nbody_set_bodies(self.h, _ptr(p), _ptr(v), _ptr(m)))
+
+    def compute_accel(self):
+        self._ck(self.lib.nbody_compute_accel(self.h))
+
+    def step(self, nsteps: int = 1):
+        self._ck(self.lib.nbody_step(self.h, int(nsteps)))
+
+    def sync(self):
+        self._ck(self.lib.nbody_sync(self.h))
+
+    def _get3(self, fn, out=None):
+        out = np.empty((self.n, 3), np.float32) if out is None else out
+        self._ck(fn(self.h, _ptr(out)))
+        return out
+
+    def get_accel(self, out=None):
+        return self._get3(self.lib.nbody_get_accel, out)
+
+    def get_positions(self, out=None):
+        return self._get3(self.lib.nbody_get_positions, out)
+
+    def get_velocities(self, out=None):
+        return self._get3(self.lib.nbody_get_velocities, out)
+
+    def get_interactions(self, out=None):
+        out = np.empty(self.n, np.uint32) if out is None else out
+        self._ck(self.lib.nbody_get_interactions(self.h, _ptr(out)))
+        return out
+
+    def get_state(self):
+        pm = np.empty((self.n, 4), np.float32)
+        vi = np.empty((self.n, 4), np.float32)
+        self._ck(self.lib.nbody_get_state(self.h, _ptr(pm), _ptr(vi)))
+        return pm, vi
+
+    def stats(self) -> dict:
+        s = _capi.nbody_stats()
+        self._ck(self.lib.nbody_get_stats(self.h, C.byref(s)))
+        return {f: getattr(s, f) for f, _ in s._fields_}
+
+    # -- debug views (parity tests) -----------------------------------------
+    def debug_keys(self):
+        out = np.empty(self.n, np.uint64)
+        self._ck(self.lib.nbody_debug_keys(self.h, _ptr(out)))
+        return out
+
+    def debug_perm(self):
+        out = np.empty(self.n, np.uint32)
+        self._ck(self.lib.nbody_debug_perm(self.h, _ptr(out)))
+        return out
+
+    def debug_level(self, level: int):
+        cnt = C.c_int64()
+        self._ck(self.lib.nbody_debug_level(self.h, int(level), C.byref(cnt), None, None, None))
+        c = cnt.value
+        pred = np.empty((c, 4), np.float64)
+        rec = np.empty((c, 4), np.float32)
+        box = np.empty((c, 6), np.float32)
+        self._ck(self.lib.nbody_debug_level(self.h, int(level), C.byref(cnt), _ptr(pred), _ptr(rec), _ptr(box)))
+        return pred, rec, box

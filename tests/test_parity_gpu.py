@@ -1,0 +1,238 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on
+the same seeded inputs.
+
+Bars: Hilbert keys and sort permutation bit-exact; BVH
+node records (fp64 com and s^2, fp32 monopole, fp32 box) bit-exact, which
+implies the north star's 1e-6 node tolerance; interaction counts per body
+equal; accelerations within 1e-4 RMS relative and 1e-2 for every body.
+"""
+import numpy as np
+import pytest
+
+from parity_utils import assert_acc_close, rel_errors
+from workloads import generate
+
+pytestmark = pytest.mark.gpu
+
+EPS = 1e-3
+DT = 1e-3
+
+
+@pytest.fixture(scope="module")
+def NB():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    from paper_conf_sc_casselldahg24_b200 import NBody
+    return NBody
+
+
+def _run_gpu(NB, pos, vel, mass, theta, key_bits, eps=EPS, traversal=0):
+    sim = NB(len(pos), theta, eps, DT, key_bits=key_bits, traversal=traversal)
+    sim.set_bodies(pos, vel, mass)
+    sim.compute_accel()
+    return sim
+
+
+def _check_pass(NB, oracle, pos, vel, mass, theta=0.5, key_bits=16, eps=EPS, targets=None, levels=True,
+                traversal=0):
+    """One force pass on both sides; returns (gpu sim, oracle result)."""
+    n = len(pos)
+    sim = _run_gpu(NB, pos, vel, mass, theta, key_bits, eps, traversal)
+    ref = oracle.step(pos, vel, mass, theta=theta, eps=eps, dt=DT, key_bits=key_bits, integrate=False,
+                      targets=targets)
+    # K2 / K3: keys and permutation bit-exact
+    assert (sim.debug_keys() == ref.keys).all()
+    assert (sim.debug_perm() == ref.perm).all()
+    # sorted state: slot order of the GPU equals the oracle's
+    pm, vi = sim.get_state()
+    assert (pm[:, :3] == ref.pos).all() and (pm[:, 3] == ref.mass).all()
+    ids = vi[:, 3].view(np.int32)
+    assert (ids == ref.ids).all()
+    # K5: node records bit-exact, every level
+    if levels:
+        for l in range(1, ref.tree.L + 1):
+            pred, rec, box = sim.debug_level(l)
+            d = ref.tree.level(l)
+            assert (pred[:, :3] == d.com).all(), f"com level {l}"
+            assert (pred[:, 3] == d.s2).all(), f"s2 level {l}"
+            assert (rec[:, :3] == d.c32).all() and (rec[:, 3] == d.m32).all(), f"rec level {l}"
+            assert (box[:, :3] == d.lo).all() and (box[:, 3:] == d.hi).all(), f"box level {l}"
+    # K6: interaction counts equal, accelerations within tolerance
+    acc_id = sim.get_accel()
+    cnt_id = sim.get_interactions()
+    tg = ref.targets
+    ids_t = ref.ids[tg]
+    assert (cnt_id[ids_t] == ref.count).all(), "interaction counts differ"
+    assert_acc_close(acc_id[ids_t], ref.acc)
+    return sim, ref
+
+
+CASES = [
+    ("uniform", 1024, 1, 0.5, 16),     # config 1
+    ("uniform", 1024, 1, 0.0, 16),     # theta = 0: direct sum
+    ("plummer", 20_000, 2, 0.5, 16),
+    ("disks", 30_001, 3, 0.5, 16),     # ragged: odd N
+    ("clustered", 25_000, 4, 0.8, 16),
+    ("clustered", 25_000, 4, 0.3, 10),  # u32 keys
+    ("plummer", 12_345, 5, 0.5, 0),    # paper grid rule (b = 5): heavy key ties
+    ("disks", 9_000, 6, 0.5, 21),      # 63-bit keys
+    ("uniform", 4097, 7, 0.5, 1),      # 3-bit keys: 8 cells, ties everywhere
+]
+
+
+@pytest.mark.parametrize("name,n,seed,theta,bits", CASES)
+def test_force_pass_parity(NB, oracle, name, n, seed, theta, bits):
+    pos, vel, mass = generate(name, n, seed)
+    _check_pass(NB, oracle, pos, vel, mass, theta=theta, key_bits=bits)
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 5, 31, 32, 33, 63, 65, 257])
+def test_small_and_ragged_n(NB, oracle, n):
+    pos, vel, mass = generate("plummer", n, 100 + n)
+    _check_pass(NB, oracle, pos, vel, mass, theta=0.5)
+
+
+def test_all_bodies_coincident(NB, oracle):
+    n = 1000
+    pos = np.tile(np.float32([0.5, -0.25, 2.0]), (n, 1))
+    vel = np.zeros_like(pos)
+    mass = np.full(n, 1.0 / n, np.float32)
+    sim, ref = _check_pass(NB, oracle, pos, vel, mass, theta=0.5, eps=1e-2)
+    assert (sim.debug_keys() == 0).all()
+
+
+def test_zero_softening_with_coincident_pairs(NB, oracle):
+    pos, vel, mass = generate("uniform", 2000, 8)
+    pos[1000:1010] = pos[0]  # coincident with body 0: r2 == 0 pairs contribute nothing
+    _check_pass(NB, oracle, pos, vel, mass, theta=0.5, eps=0.0)
+
+
+def test_mixed_masses(NB, oracle):
+    pos, vel, _ = generate("clustered", 8000, 9)
+    mass = np.random.default_rng(9).lognormal(0.0, 1.0, 8000).astype(np.float32)
+    _check_pass(NB, oracle, pos, vel, mass, theta=0.6)
+
+
+def test_traversal_variants_agree(NB, oracle):
+    pos, vel, mass = generate("disks", 20_000, 10)
+    s0 = _run_gpu(NB, pos, vel, mass, 0.5, 16, traversal=0)
+    s1 = _run_gpu(NB, pos, vel, mass, 0.5, 16, traversal=1)
+    assert (s0.get_interactions() == s1.get_interactions()).all()
+    e = rel_errors(s0.get_accel(), s1.get_accel())
+    assert e.max() < 1e-5
+
+
+def test_step_parity_and_determinism(NB, oracle):
+    """One full step (force + leapfrog) against the oracle; two GPU runs are
+    bit-identical (no float atomics anywhere); graph == plain launches."""
+    pos, vel, mass = generate("plummer", 50_000, 11)
+    outs = []
+    for graph in (True, False, True):
+        sim = NB(len(pos), 0.5, EPS, DT, key_bits=16, use_graph=graph)
+        sim.set_bodies(pos, vel, mass)
+        sim.step(1)
+        outs.append((sim.get_positions(), sim.get_velocities(), sim.get_accel()))
+    for o in outs[1:]:
+        for a, b in zip(outs[0], o):
+            assert (a == b).all()
+    ref = oracle.step(pos, vel, mass, theta=0.5, eps=EPS, dt=DT, key_bits=16)
+    x_gpu, v_gpu, a_gpu = outs[0]
+    order = ref.ids
+    assert_acc_close(a_gpu[order], ref.acc)
+    # v = v0 + a dt; positions move by v dt: differences are a-rounding sized
+    dv = np.abs(v_gpu[order].astype(float) - ref.vel.astype(float)).max()
+    assert dv <= 1e-2 * DT * np.abs(ref.acc).max() + 1e-6 * np.abs(ref.vel).max()
+    dx = np.abs(x_gpu[order].astype(float) - ref.pos.astype(float)).max()
+    assert dx <= 2 * np.spacing(np.abs(ref.pos).max().astype(np.float32)) + DT * dv
+
+
+def test_ten_steps_track_the_oracle(NB, oracle):
+    """10 steps (config 2's loop, small N): trajectories stay within the
+    drift the tolerances allow."""
+    n, steps = 20_000, 10
+    pos, vel, mass = generate("plummer", n, 12)
+    sim = NB(n, 0.5, EPS, DT, key_bits=16)
+    sim.set_bodies(pos, vel, mass)
+    sim.step(steps)
+    xg = sim.get_positions()
+    x, v, m, ids = pos, vel, mass, np.arange(n)
+    amax = 0.0
+    for _ in range(steps):
+        r = oracle.step(x, v, m, ids, theta=0.5, eps=EPS, dt=DT, key_bits=16)
+        x, v, m, ids = r.pos, r.vel, r.mass, r.ids
+        amax = max(amax, float(np.abs(r.acc).max()))
+    xo = np.empty_like(x)
+    xo[ids] = x
+    # |dx| <= steps^2 dt^2 max|da| with |da| <= 1e-2 |a| per body and step,
+    # plus fp32 rounding of the positions each step
+    bound = steps * steps * DT * DT * 1e-2 * amax + steps * 2 * np.spacing(np.float32(np.abs(x).max()))
+    assert np.abs(xg.astype(float) - xo.astype(float)).max() <= bound
+    st = sim.stats()
+    assert st["steps"] == steps and st["interactions"] > 0
+
+
+def test_device_pointers_round_trip(NB):
+    import torch
+    pos, vel, mass = generate("uniform", 5000, 13)
+    tp, tv, tm = (torch.from_numpy(a).cuda() for a in (pos, vel, mass))
+    sim = NB(5000, 0.5, EPS, DT)
+    sim.set_bodies(tp, tv, tm)
+    out = torch.empty((5000, 3), dtype=torch.float32, device="cuda")
+    sim.get_positions(out)
+    assert (out.cpu().numpy() == pos).all()
+    sim.compute_accel()
+    a_host = sim.get_accel()
+    sim.get_accel(out)
+    assert (out.cpu().numpy() == a_host).all()
+
+
+def test_invalid_bodies_rejected(NB):
+    from paper_conf_sc_casselldahg24_b200 import NBodyError
+    pos, vel, mass = generate("uniform", 100, 14)
+    sim = NB(100, 0.5, EPS, DT)
+    bad = mass.copy()
+    bad[5] = 0.0
+    with pytest.raises(NBodyError):
+        sim.set_bodies(pos, vel, bad)
+    pos2 = pos.copy()
+    pos2[3, 1] = np.nan
+    with pytest.raises(NBodyError):
+        sim.set_bodies(pos2, vel, mass)
+    with pytest.raises(NBodyError):
+        sim.step(1)  # nothing loaded
+    sim.set_bodies(pos, vel, mass)
+    sim.step(1)
+
+
+# ---------------------------------------------------------------- full size --
+def _sampled_full_size(NB, oracle, name, n, seed, nsample):
+    pos, vel, mass = generate(name, n, seed)
+    sim = NB(n, 0.5, EPS, DT, key_bits=16)
+    sim.set_bodies(pos, vel, mass)
+    sim.compute_accel()
+    rng = np.random.default_rng(seed)
+    targets = np.sort(rng.choice(n, nsample, replace=False))
+    ref = oracle.step(pos, vel, mass, theta=0.5, eps=EPS, dt=DT, key_bits=16, integrate=False, targets=targets)
+    assert (sim.debug_keys() == ref.keys).all()
+    assert (sim.debug_perm() == ref.perm).all()
+    # node records: the top 8 levels entirely, sampled nodes below
+    for l in range(1, ref.tree.L + 1):
+        pred, rec, box = sim.debug_level(l)
+        d = ref.tree.level(l)
+        sel = slice(None) if len(pred) <= 4096 else rng.choice(len(pred), 4096, replace=False)
+        assert (pred[sel, :3] == d.com[sel]).all() and (pred[sel, 3] == d.s2[sel]).all()
+        assert (rec[sel, :3] == d.c32[sel]).all() and (rec[sel, 3] == d.m32[sel]).all()
+    acc = sim.get_accel()
+    cnt = sim.get_interactions()
+    ids_t = ref.ids[targets]
+    assert (cnt[ids_t] == ref.count).all()
+    assert_acc_close(acc[ids_t], ref.acc)
+
+
+def test_config2_plummer_1M_sampled(NB, oracle):
+    _sampled_full_size(NB, oracle, "plummer", 1_000_000, 2, 3000)
+
+
+@pytest.mark.slow
+def test_config3_disks_10M_sampled(NB, oracle):
+    _sampled_full_size(NB, oracle, "disks", 10_000_000, 3, 2000)
