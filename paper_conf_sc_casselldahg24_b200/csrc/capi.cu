@@ -114,32 +114,33 @@ int resolve_bits(int64_t n, int opt) {
 
 size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
 
-// Tree plan: levels, counts, offsets (sizes follow from N alone).
+// Tree plan (sizes follow from N alone).  Heap numbering: node
+// (l, j) has global id g = 2^(L-l) + j, so the root is 1, the children of g
+// are 2g and 2g+1 and leaf i is 2^L + i; level l only uses its first
+// ceil(N / 2^l) ids.  Returns the number of ids (2^(L+1)).
 int64_t plan_tree(TreeView& t, int64_t n) {
   t.n = n;
   t.L = 0;
   while ((int64_t(1) << t.L) < n) ++t.L;
   t.count[0] = n;
-  t.off[0] = 0;
-  int64_t total = 0;
+  t.off[0] = int64_t(1) << t.L;
   for (int l = 1; l <= t.L; ++l) {
     t.count[l] = (t.count[l - 1] + 1) / 2;
-    t.off[l] = total;
-    total += (t.count[l] + 1) & ~int64_t(1);  // keep sibling pairs aligned
+    t.off[l] = int64_t(1) << (t.L - l);
   }
   for (int l = t.L + 1; l < kMaxLevels; ++l) t.count[l] = t.off[l] = 0;
-  return total;
+  return int64_t(2) << t.L;
 }
 
 nbody_status allocate(nbody_ctx* c) {
   const int64_t n = c->n;
-  const int64_t nodes = plan_tree(c->tree, n);
+  const int64_t ids = plan_tree(c->tree, n);   // rec / s2f cover leaves too
+  const int64_t inner = ids / 2;                // pred / mom / box: internal ids < 2^L
   c->nbbox = 2 * c->nsm;
   const int64_t tiles = sort_tiles(n);
   size_t sz[32];
   int k = 0;
   sz[k++] = 16 * size_t(n);                         // pm0
-  sz[k++] = 16 * size_t(n);                         // pm1
   sz[k++] = 16 * size_t(n);                         // vi0
   sz[k++] = 16 * size_t(n);                         // vi1
   sz[k++] = 8 * size_t(n);                          // keys0
@@ -155,11 +156,12 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 8;                                      // total
   sz[k++] = 8;                                      // bad
   sz[k++] = sort_scratch_bytes(n);                  // sort
-  sz[k++] = 32 * size_t(nodes);                     // pred
-  sz[k++] = 16 * size_t(nodes);                     // rec
-  sz[k++] = 32 * size_t(nodes);                     // mom
-  sz[k++] = 16 * size_t(nodes);                     // blo
-  sz[k++] = 16 * size_t(nodes);                     // bhi
+  sz[k++] = 32 * size_t(inner);                     // pred
+  sz[k++] = 16 * size_t(ids);                       // rec (leaf ids hold the sorted bodies)
+  sz[k++] = 32 * size_t(inner);                     // mom
+  sz[k++] = 16 * size_t(inner);                     // blo
+  sz[k++] = 16 * size_t(inner);                     // bhi
+  sz[k++] = 8 * size_t(ids);                        // rc (-inf at the leaves)
   size_t total = 0;
   for (int i = 0; i < k; ++i) total += align_up(sz[i]);
   cudaError_t e = cudaMalloc(&c->arena, total);
@@ -172,7 +174,6 @@ nbody_status allocate(nbody_ctx* c) {
   int i = 0;
   auto take = [&](void) -> char* { char* r = p; p += align_up(sz[i++]); return r; };
   c->pm[0] = (float4*)take();
-  c->pm[1] = (float4*)take();
   c->vi[0] = (float4*)take();
   c->vi[1] = (float4*)take();
   c->keys[0] = take();
@@ -193,6 +194,16 @@ nbody_status allocate(nbody_ctx* c) {
   c->tree.mom = (double4*)take();
   c->tree.blo = (float4*)take();
   c->tree.bhi = (float4*)take();
+  c->tree.rc = (float2*)take();
+  c->tree.grid = c->grid;
+  c->tree.th2 = c->theta * c->theta;
+  // the sorted bodies live in the leaf ids of the record array
+  c->pm[1] = c->tree.rec + (int64_t(1) << c->tree.L);
+  // leaves always interact when reached: thresholds (-inf, -inf), set once
+  const float ninf = -INFINITY;
+  launch_fill_float2(c->tree.rc + (int64_t(1) << c->tree.L), n, make_float2(ninf, ninf), nullptr);
+  e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
   c->sort.n = n;
   c->sort.tiles = tiles;
   c->sort.ghist = (uint32_t*)sortmem;
@@ -235,6 +246,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   ForceParams fp;
   fp.t = c->tree;
   fp.leaves = c->pm[1];
+  fp.grid = c->grid;
   fp.t_begin = 0;
   fp.t_end = n;
   fp.th2 = c->theta * c->theta;

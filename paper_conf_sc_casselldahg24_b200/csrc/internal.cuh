@@ -19,7 +19,8 @@ struct GridInfo {
   float hi[3];
   double inv;    // 2^b / ext, or 0 when ext == 0 [A17]
   int b;         // bits per axis
-  int pad;
+  float abs_d2;  // absolute slack of the fp32 opening-test filter: 1e-9 R^2,
+                 // R = max |coordinate| (K6)
 };
 
 // Balanced, ragged BVH stored level by level ([A6]).  Level 0 is the
@@ -33,6 +34,12 @@ struct TreeView {
   int64_t off[kMaxLevels];     // start of level l in the node arrays
   double4* pred;   // (com64 x, y, z, s^2)   opening test data, fp64 [A3][A16]
   float4* rec;     // ((float)com64, (float)M) monopole for the interaction
+  float2* rc;      // (lo, hi) fp32 thresholds on |c32 - x|^2 of the filtered
+                   // opening test: d2 < lo => open, d2 > hi => accept, else
+                   // the exact fp64 test; leaves
+                   // hold (-inf, -inf)
+  const GridInfo* grid;  // bbox of this step (filter slack)
+  double th2;            // theta^2 the thresholds were built for
   double4* mom;    // (M, Mx, My, Mz) fp64 moments (build only) [A12]
   float4* blo;     // AABB lo (x, y, z, -)
   float4* bhi;     // AABB hi (x, y, z, -)
@@ -41,6 +48,7 @@ struct TreeView {
 struct ForceParams {
   TreeView t;
   const float4* leaves;   // sorted (x, y, z, m)
+  const GridInfo* grid;   // this step's bbox (for the fp32 filter slack)
   int64_t t_begin;        // owned target slots [t_begin, t_end)
   int64_t t_end;
   double th2;             // theta^2 (fp64, used by the opening test)
@@ -83,6 +91,7 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // ---- K7 and helpers --------------------------------------------------------
 void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
                      float4* vi_out, cudaStream_t s);
+void launch_fill_float2(float2* p, int64_t count, float2 v, cudaStream_t s);
 void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
                         int* bad, cudaStream_t s);
 // out[id][3] <- src[slot].xyz for slots [0, n); id from vi[slot].w

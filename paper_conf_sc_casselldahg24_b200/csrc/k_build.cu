@@ -34,7 +34,22 @@ __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, dou
   double s = __dsub_rn(double(hi.x), double(lo.x));
   s = fmax(s, __dsub_rn(double(hi.y), double(lo.y)));
   s = fmax(s, __dsub_rn(double(hi.z), double(lo.z)));
-  t.pred[node] = make_double4(cx, cy, cz, __dmul_rn(s, s));
+  const double s2 = __dmul_rn(s, s);
+  t.pred[node] = make_double4(cx, cy, cz, s2);
+  // Filter thresholds on the fp32 squared distance (DESIGN.md "fp32
+  // filter"): |d2_fp32 - d^2| <= 1.01e-4 d^2 + A with A = 1e-9 R^2, so
+  // d2 > (1 + 2e-4) s^2/theta^2 + A surely accepts and
+  // d2 < (1 - 2e-4) s^2/theta^2 - A surely opens.
+  float2 rc;
+  if (t.th2 > 0.0) {
+    const double q = s2 / t.th2;
+    const double A = double(t.grid->abs_d2);
+    rc.x = __double2float_rd((1.0 - 2e-4) * q - A);
+    rc.y = __double2float_ru((1.0 + 2e-4) * q + A);
+  } else {  // theta = 0 opens every node
+    rc.x = rc.y = __int_as_float(0x7f800000);
+  }
+  t.rc[node] = rc;
   t.rec[node] = make_float4(__double2float_rn(cx), __double2float_rn(cy), __double2float_rn(cz), __double2float_rn(M));
 }
 

@@ -6,19 +6,42 @@
 // opening test for k and n passes it (or n is a leaf other than k).  The
 // opening test is the fixed fp64 expression [A3][A16][A20]
 //     s^2 < theta^2 * fma(dz, dz, fma(dy, dy, dx*dx)),  d = com64 - x_k,
-// evaluated with explicitly rounded intrinsics, so every decision -- hence
-// every interaction list -- is bit-identical to the oracle's.  The
-// interaction itself is fp32 (rsqrtf + FMA) on the monopole
-// ((float)com, (float)M); its summation order is free (tolerance-checked).
+// so every decision -- hence every interaction list -- is bit-identical to
+// the oracle's.  The interaction itself is fp32 (MUFU rsqrt + FMA) on the
+// monopole ((float)com, (float)M); its summation order is free
+// (tolerance-checked).  Interactions with r == 0 (the target itself, or a
+// coincident body when eps == 0) add exactly 0.
 //
-// Variant 1, warp mask-stack walk: the 32 lanes of a warp own 32
-// Hilbert-consecutive targets and walk the tree together.  A shared-memory
-// stack holds sibling pairs (level, pair index, lane mask of the lanes that
-// reached the pair).  Each popped pair is loaded once for the whole warp
-// (broadcast), every lane in the mask tests both siblings, lanes that accept
-// interact immediately, and the ballots of rejecting lanes become the masks
-// of the children pairs.  No lane ever visits a node it would not visit in
-// its own DFS, so lists are exact; idle lanes cost issue slots only.
+// Tree addressing: heap ids (capi.cu plan_tree): root 1, children of g are
+// 2g and 2g+1, leaf i is 2^L + i, level of g is L - floor(log2 g).  rec[g]
+// is the fp32 monopole (the sorted body for a leaf), rc[g] the fp32 filter
+// thresholds on the squared distance, pred[g] the exact fp64 (com, s^2) of
+// an internal node.
+//
+// Variant 0 (default), group-classified walk.  A warp owns 32
+// Hilbert-consecutive targets with bounding box B.
+//   A. Lanes classify 32 tree nodes at a time against B with exact fp64
+//      bounds of the opening test over all of B: SURE_ACCEPT (every lane
+//      accepts: the node joins the warp's common list), SURE_REJECT (every
+//      lane opens it: its children are classified next) or MIXED.  Leaves
+//      reached here are common too.  Every node reaching A has been opened
+//      by every lane, so common entries are in every lane's list.
+//   B. The common list is evaluated densely: each entry is read once from
+//      shared memory (broadcast) and every lane interacts with it.
+//   C. Each MIXED node is walked with the per-lane mask stack below,
+//      starting with all lanes.
+// Variant 1, the mask-stack walk from the root for every warp.
+//
+// Mask stack: a warp-uniform DFS stack of (sibling pair, mask of the lanes
+// that reached it), held in registers (lane i holds entry i; depth <= L+1 <
+// 32).  Each popped pair is loaded once for the warp (one 32-byte load),
+// lanes in the mask test both siblings, accepting lanes interact, and the
+// ballots of opening lanes become the masks of the children pairs.  No lane
+// ever visits a node outside its own DFS, so lists are exact.
+//
+// Per-lane opening decisions use an fp32 filter with a rigorous error bound
+// and fall back to the exact fp64 expression inside the uncertainty band
+// (DESIGN.md "fp32 filter"), so they equal the fp64 decisions.
 #include "internal.cuh"
 
 namespace nb {
@@ -26,7 +49,21 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 
-__device__ __forceinline__ bool opening_accept(const double4& p, double x, double y, double z, double th2) {
+__device__ __forceinline__ float rsqrt_fast(float x) {
+  float y;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+// One 32-byte load of a sibling pair of records (g even => 32-B aligned).
+__device__ __forceinline__ void load_pair(const float4* p, float4& a, float4& b) {
+  asm volatile("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+               : "l"(p));
+}
+
+// Exact fp64 opening test (the definition).
+__device__ __forceinline__ bool opening_accept64(const double4& p, double x, double y, double z, double th2) {
   const double dx = __dsub_rn(p.x, x);
   const double dy = __dsub_rn(p.y, y);
   const double dz = __dsub_rn(p.z, z);
@@ -34,105 +71,410 @@ __device__ __forceinline__ bool opening_accept(const double4& p, double x, doubl
   return p.w < __dmul_rn(th2, d2);
 }
 
+struct Target {
+  float x, y, z;    // the lane's target position
+  float eps2;
+  double th2;
+};
+
 struct Acc {
   float x = 0.f, y = 0.f, z = 0.f;
   uint32_t n = 0;
-  __device__ __forceinline__ void add(const float4& s, const float4& me, float eps2) {
-    const float dx = s.x - me.x, dy = s.y - me.y, dz = s.z - me.z;
-    const float r2 = fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2)));
-    const float inv = r2 > 0.f ? rsqrtf(r2) : 0.f;  // r2 == 0 only when eps == 0: no contribution
-    const float w = s.w * inv * inv * inv;
+  // add m r / (|r|^2 + eps^2)^(3/2) when `on`; d2 = |r|^2 already computed
+  __device__ __forceinline__ void add(bool on, float dx, float dy, float dz, float d2, float m, float eps2) {
+    const float r2 = d2 + eps2;
+    const float inv = r2 > 0.f ? rsqrt_fast(r2) : 0.f;
+    const float w = on ? m * inv * inv * inv : 0.f;
     x = fmaf(w, dx, x);
     y = fmaf(w, dy, y);
     z = fmaf(w, dz, z);
-    ++n;
   }
 };
 
-constexpr int kWarpsPerBlock = 8;
-constexpr int kStack = 64;
+struct Probe {
+  float dx, dy, dz, d2;
+};
 
-__global__ __launch_bounds__(32 * kWarpsPerBlock) void k_force_maskstack(const ForceParams P) {
-  __shared__ uint32_t s_idx[kWarpsPerBlock][kStack];
-  __shared__ uint32_t s_msk[kWarpsPerBlock][kStack];
-  __shared__ int s_lvl[kWarpsPerBlock][kStack];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t k = P.t_begin + (int64_t(blockIdx.x) * kWarpsPerBlock + w) * 32 + lane;
-  const bool active = k < P.t_end;
-  const uint32_t amask = __ballot_sync(kFull, active);
-  if (amask == 0) return;
-  const float4 me = active ? P.leaves[k] : make_float4(0.f, 0.f, 0.f, 0.f);
-  const double x64 = me.x, y64 = me.y, z64 = me.z;
-  Acc a;
-  const int L = P.t.L;
+__device__ __forceinline__ Probe probe(const float4& r, const Target& T) {
+  Probe p;
+  p.dx = r.x - T.x;
+  p.dy = r.y - T.y;
+  p.dz = r.z - T.z;
+  p.d2 = fmaf(p.dz, p.dz, fmaf(p.dy, p.dy, p.dx * p.dx));
+  return p;
+}
 
-  int sp = 1;
-  if (lane == 0) {
-    s_lvl[w][0] = L;
-    s_idx[w][0] = 0;
-    s_msk[w][0] = amask;
+// Loop invariants of the walk, pinned in registers.
+struct Walk {
+  const float4* rec;
+  const float4* rc2;     // rc viewed as pairs (lo_A, hi_A, lo_B, hi_B)
+  const float2* rc;
+  const double4* pred;
+  uint32_t leaf0, n;
+  int L;
+};
+
+template <class T>
+__device__ __forceinline__ T* in_reg(T* p) {
+  asm volatile("" : "+l"(p));
+  return p;
+}
+
+__device__ __forceinline__ Walk make_walk(const ForceParams& P) {
+  Walk W;
+  W.rec = in_reg(P.t.rec);
+  W.rc = in_reg(P.t.rc);
+  W.rc2 = reinterpret_cast<const float4*>(W.rc);
+  W.pred = in_reg(P.t.pred);
+  W.L = P.t.L;
+  W.leaf0 = 1u << W.L;
+  W.n = uint32_t(P.t.n);
+  return W;
+}
+
+// Per-lane decision for one internal node: fp32 filter, fp64 fallback.
+__device__ __forceinline__ bool decide1(const Walk& W, uint32_t g, bool in, float d2, float2 c, const Target& T) {
+  bool acc = in && d2 > c.y;
+  const bool und = in && !acc && !(d2 < c.x);
+  if (__any_sync(kFull, und)) {
+    if (und) acc = opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
   }
-  __syncwarp();
+  return acc;
+}
+
+// The per-lane mask-stack walk of the subtree of node g0 for the lanes in
+// mask0 (all of which reached g0).
+__device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32_t kid, Acc& a, int lane, uint32_t g0,
+                                          uint32_t mask0) {
+  // the start node on its own
+  {
+    const bool in = (mask0 >> lane) & 1u;
+    const float4 r = __ldg(W.rec + g0);
+    const Probe p = probe(r, T);
+    if (g0 >= W.leaf0) {  // a leaf (N == 1 root)
+      const bool acc = in && g0 != kid;
+      a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+      a.n += acc;
+      return;
+    }
+    const bool acc = decide1(W, g0, in, p.d2, __ldg(W.rc + g0), T);
+    if (__any_sync(kFull, acc)) a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+    a.n += acc;
+    const uint32_t rej = __ballot_sync(kFull, in && !acc);
+    if (rej == 0) return;
+    mask0 = rej;
+    g0 = 2u * g0;
+  }
+  // sibling pairs; lane i holds stack entry i (depth <= L + 1 < 32)
+  uint32_t sg = g0, sm = mask0;
+  int sp = 1;
   while (sp > 0) {
     --sp;
-    const int l = s_lvl[w][sp];
-    const uint32_t p = s_idx[w][sp];
-    const uint32_t m = s_msk[w][sp];
-    __syncwarp();
-    const bool in = (m >> lane) & 1u;
-    const int64_t jA = 2 * int64_t(p), jB = jA + 1;
-    const bool hasB = jB < P.t.count[l];
-    if (l == 0) {  // two leaves: exact interactions, the target excluded
-      const float4 A = P.leaves[jA];
-      if (in && jA != k) a.add(A, me, P.eps2);
-      if (hasB) {
-        const float4 B = P.leaves[jB];
-        if (in && jB != k) a.add(B, me, P.eps2);
+    const uint32_t g = __shfl_sync(kFull, sg, sp);
+    const uint32_t em = __shfl_sync(kFull, sm, sp);
+    const int l = W.L - 31 + __clz(int(g));
+    const bool in = (em >> lane) & 1u;
+    const bool hasB = (((g + 1u) << l) - W.leaf0) < W.n;  // right sibling exists iff its first leaf < N
+    float4 rA, rB;
+    load_pair(W.rec + g, rA, rB);
+    const Probe pA = probe(rA, T);
+    const Probe pB = probe(rB, T);
+    bool accA, accB;
+    if (l == 0) {  // leaves: exact interactions, the target itself excluded
+      accA = in && g != kid;
+      accB = in && hasB && g + 1u != kid;
+    } else {
+      const float4 c = __ldg(W.rc2 + (g >> 1));
+      accA = in && pA.d2 > c.y;
+      accB = in && hasB && pB.d2 > c.w;
+      const bool undA = in && !accA && !(pA.d2 < c.x);
+      const bool undB = in && hasB && !accB && !(pB.d2 < c.z);
+      if (__any_sync(kFull, undA || undB)) {  // rare: exact fp64 decision
+        if (undA) accA = opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
+        if (undB) accB = opening_accept64(W.pred[g + 1], T.x, T.y, T.z, T.th2);
       }
-      continue;
+      const uint32_t rejB = __ballot_sync(kFull, in && hasB && !accB);
+      const uint32_t rejA = __ballot_sync(kFull, in && !accA);
+      // push the children pair of B, then of A (A's subtree is walked first)
+      const bool pushB = rejB != 0, pushA = rejA != 0;
+      if (pushB && lane == sp) { sg = 2u * g + 2u; sm = rejB; }
+      const int q = sp + int(pushB);
+      if (pushA && lane == q) { sg = 2u * g; sm = rejA; }
+      sp = q + int(pushA);
     }
-    const int64_t node = P.t.off[l] + jA;
-    const double4 pa = P.t.pred[node];
-    const bool accA = opening_accept(pa, x64, y64, z64, P.th2);
-    bool accB = false;
-    if (hasB) accB = opening_accept(P.t.pred[node + 1], x64, y64, z64, P.th2);
-    const uint32_t rejA = __ballot_sync(kFull, in && !accA);
-    const uint32_t rejB = __ballot_sync(kFull, in && hasB && !accB);
-    const bool doA = in && accA, doB = in && hasB && accB;
-    if (__any_sync(kFull, doA)) {
-      const float4 r = P.t.rec[node];
-      if (doA) a.add(r, me, P.eps2);
-    }
-    if (__any_sync(kFull, doB)) {
-      const float4 r = P.t.rec[node + 1];
-      if (doB) a.add(r, me, P.eps2);
-    }
-    // children of (l, jB) then of (l, jA): the A subtree is walked first
-    if (lane == 0) {
-      int q = sp;
-      if (rejB) { s_lvl[w][q] = l - 1; s_idx[w][q] = uint32_t(jB); s_msk[w][q] = rejB; ++q; }
-      if (rejA) { s_lvl[w][q] = l - 1; s_idx[w][q] = uint32_t(jA); s_msk[w][q] = rejA; }
-    }
-    sp += (rejB != 0) + (rejA != 0);
-    __syncwarp();
+    if (__any_sync(kFull, accA)) a.add(accA, pA.dx, pA.dy, pA.dz, pA.d2, rA.w, T.eps2);
+    if (__any_sync(kFull, accB)) a.add(accB, pB.dx, pB.dy, pB.dz, pB.d2, rB.w, T.eps2);
+    a.n += accA;
+    a.n += accB;
   }
+}
+
+__device__ __forceinline__ Target load_target(const ForceParams& P, int64_t k, bool active) {
+  Target T;
+  const float4 me = active ? P.leaves[k] : make_float4(0.f, 0.f, 0.f, 0.f);
+  T.x = me.x;
+  T.y = me.y;
+  T.z = me.z;
+  T.th2 = P.th2;
+  T.eps2 = P.eps2;
+  return T;
+}
+
+__device__ __forceinline__ void store_result(const ForceParams& P, int64_t k, bool active, const Acc& a, int lane) {
   if (active) {
     P.acc[k - P.t_begin] = make_float4(a.x, a.y, a.z, 0.f);
     P.count[k - P.t_begin] = a.n;
   }
-  const uint32_t tot = __reduce_add_sync(kFull, a.n);
+  const uint32_t tot = __reduce_add_sync(kFull, active ? a.n : 0u);
   if (lane == 0) atomicAdd(P.total, (unsigned long long)tot);
+}
+
+// ------------------------------------------------------------ variant 1 ----
+constexpr int kV1Warps = 8;
+
+__global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForceParams P) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t k = P.t_begin + (int64_t(blockIdx.x) * kV1Warps + w) * 32 + lane;
+  const bool active = k < P.t_end;
+  const uint32_t amask = __ballot_sync(kFull, active);
+  if (amask == 0) return;
+  const Target T = load_target(P, k, active);
+  Acc a;
+  const Walk W = make_walk(P);
+  const uint32_t kid = W.leaf0 + uint32_t(k);
+  mask_walk(W, T, kid, a, lane, 1u, amask);
+  store_result(P, k, active, a, lane);
+}
+
+// ------------------------------------------------------------ variant 0 ----
+constexpr int kV0Warps = 4;
+constexpr int kCapA = 256;  // box-phase stack (ids)
+constexpr int kCapT = 512;  // transposed-phase stack (id, mask)
+constexpr int kCapD = 128;  // dense list (record, mask)
+
+struct V0Smem {
+  float4 tgt[32];       // the warp's target positions
+  float4 drec[kCapD];   // dense list: monopole / body record
+  uint32_t dmsk[kCapD]; //             lanes that interact with it
+  uint32_t astk[kCapA];
+  uint2 tstk[kCapT];    // (id, mask of the targets that reached it)
+};
+
+__device__ __forceinline__ float warp_minf(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fminf(v, __shfl_xor_sync(kFull, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_maxf(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(kFull, v, o));
+  return v;
+}
+
+// Dense list: entry e interacts with the lanes in dmsk[e].
+__device__ __forceinline__ void dense(const V0Smem& S, int nd, const Target& T, Acc& a, int lane) {
+#pragma unroll 4
+  for (int e = 0; e < nd; ++e) {
+    const float4 s = S.drec[e];
+    const bool on = (S.dmsk[e] >> lane) & 1u;
+    const Probe p = probe(s, T);
+    a.add(on, p.dx, p.dy, p.dz, p.d2, s.w, T.eps2);
+    a.n += on;
+  }
+}
+
+__global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForceParams P) {
+  __shared__ V0Smem s_all[kV0Warps];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  V0Smem& S = s_all[w];
+  const int64_t k0 = P.t_begin + (int64_t(blockIdx.x) * kV0Warps + w) * 32;
+  const int64_t k = k0 + lane;
+  const bool active = k < P.t_end;
+  const uint32_t amask = __ballot_sync(kFull, active);
+  if (amask == 0) return;
+  const Target T = load_target(P, k, active);
+  Acc a;
+  const uint32_t lt = (1u << lane) - 1u;
+  const Walk W = make_walk(P);
+  const uint32_t leaf0 = W.leaf0;
+  const uint32_t n = W.n;
+  const int L = W.L;
+  const uint32_t kid = leaf0 + uint32_t(k);
+  const uint32_t kid0 = leaf0 + uint32_t(k0);
+  S.tgt[lane] = make_float4(T.x, T.y, T.z, 0.f);
+
+  // group box over the active lanes (exact fp32 min/max, used in fp64)
+  const float inf = __int_as_float(0x7f800000);
+  const double blx = warp_minf(active ? T.x : inf), bhx = warp_maxf(active ? T.x : -inf);
+  const double bly = warp_minf(active ? T.y : inf), bhy = warp_maxf(active ? T.y : -inf);
+  const double blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
+
+  int na = 1, nt = 0, nd = 0;
+  if (lane == 0) S.astk[0] = 1u;
+  __syncwarp();
+
+  while (true) {
+    if (nt >= 32 || (na == 0 && nt > 0)) {
+      // ---- T: transposed classification of up to 32 (node, mask) entries
+      const int take = nt < 32 ? nt : 32;
+      const int base = nt - take;
+      const bool has = lane < take;
+      const uint2 e = has ? S.tstk[base + lane] : make_uint2(leaf0, 0u);
+      __syncwarp();
+      nt = base;
+      const uint32_t g = e.x, m = e.y;
+      const float4 r = __ldg(W.rec + g);
+      const float2 c = __ldg(W.rc + g);  // leaves: (-inf, -inf): always interact
+      uint32_t am = 0u, rm = 0u;
+#pragma unroll
+      for (int t = 0; t < 32; ++t) {
+        const float4 tp = S.tgt[t];
+        const float dx = r.x - tp.x, dy = r.y - tp.y, dz = r.z - tp.z;
+        const float d2 = fmaf(dz, dz, fmaf(dy, dy, dx * dx));
+        am |= d2 > c.y ? (1u << t) : 0u;
+        rm |= d2 < c.x ? (1u << t) : 0u;
+      }
+      am &= m;
+      rm &= m;
+      uint32_t und = m & ~(am | rm);
+      if (__any_sync(kFull, und != 0u)) {  // rare: exact fp64 decisions
+        if (und) {
+          const double4 pd = W.pred[g];
+          do {
+            const int t = __ffs(int(und)) - 1;
+            const float4 tp = S.tgt[t];
+            if (opening_accept64(pd, tp.x, tp.y, tp.z, T.th2)) am |= 1u << t; else rm |= 1u << t;
+            und &= und - 1u;
+          } while (und);
+        }
+      }
+      if (g >= leaf0 && g - kid0 < 32u) am &= ~(1u << (g - kid0));  // a leaf never acts on itself
+      // dense-list append
+      const uint32_t bd = __ballot_sync(kFull, am != 0u);
+      if (am) {
+        const int pos = nd + __popc(bd & lt);
+        S.drec[pos] = r;
+        S.dmsk[pos] = am;
+      }
+      nd += __popc(bd);
+      // children of opened nodes, with the mask of the targets that opened them
+      const int l = L - 31 + __clz(int(g));
+      const bool two = rm && (((2u * g + 1u) << (l - 1)) - leaf0) < n;
+      const bool room = nt + 64 <= kCapT;
+      const bool push = rm != 0u && room;
+      const uint32_t b1 = __ballot_sync(kFull, push);
+      const uint32_t b2 = __ballot_sync(kFull, push && two);
+      if (push) {
+        const int pos = nt + __popc(b1 & lt) + __popc(b2 & lt);
+        S.tstk[pos] = make_uint2(2u * g, rm);
+        if (two) S.tstk[pos + 1] = make_uint2(2u * g + 1u, rm);
+      }
+      nt += __popc(b1) + __popc(b2);
+      __syncwarp();
+      if (nd > kCapD - 32) {
+        dense(S, nd, T, a, lane);
+        nd = 0;
+        __syncwarp();
+      }
+      // no room (never observed at the sizes we run): walk those subtrees per lane
+      uint32_t spill = __ballot_sync(kFull, rm != 0u && !room);
+      while (spill) {
+        const int src = __ffs(int(spill)) - 1;
+        spill &= spill - 1u;
+        const uint32_t gs = __shfl_sync(kFull, g, src);
+        const uint32_t ms = __shfl_sync(kFull, rm, src);
+        mask_walk(W, T, kid, a, lane, 2u * gs, ms);
+        // (the walk starts at the left child; the right child, if any:)
+        const int ls = L - 31 + __clz(int(gs));
+        if ((((2u * gs + 1u) << (ls - 1)) - leaf0) < n) mask_walk(W, T, kid, a, lane, 2u * gs + 1u, ms);
+      }
+    } else if (na > 0) {
+      // ---- A: box classification of up to 32 nodes reached by every lane
+      const int take = na < 32 ? na : 32;
+      const int base = na - take;
+      const bool has = lane < take;
+      const uint32_t g = has ? S.astk[base + lane] : 0u;
+      __syncwarp();
+      na = base;
+      const bool guard = na + 64 > kCapA;
+      int cls = 0;  // 1 dense (all lanes), 2 expand, 3 transposed
+      float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
+      bool two = false;
+      if (has) {
+        if (g >= leaf0) {
+          cls = 1;
+          r = __ldg(W.rec + g);
+        } else {
+          const double4 p = W.pred[g];
+          // exact bounds of |com - x|^2 over the box
+          const double ax0 = __dsub_rn(blx, p.x), ax1 = __dsub_rn(p.x, bhx);
+          const double ay0 = __dsub_rn(bly, p.y), ay1 = __dsub_rn(p.y, bhy);
+          const double az0 = __dsub_rn(blz, p.z), az1 = __dsub_rn(p.z, bhz);
+          const double nx = fmax(0.0, fmax(ax0, ax1)), ny = fmax(0.0, fmax(ay0, ay1)),
+                       nz = fmax(0.0, fmax(az0, az1));
+          const double fx = fmax(fabs(ax0), fabs(ax1)), fy = fmax(fabs(ay0), fabs(ay1)),
+                       fz = fmax(fabs(az0), fabs(az1));
+          const double dmin2 = nx * nx + ny * ny + nz * nz;
+          const double dmax2 = fx * fx + fy * fy + fz * fz;
+          if (p.w < T.th2 * dmin2 * (1.0 - 1e-12)) {
+            cls = 1;
+            r = __ldg(W.rec + g);
+          } else if (p.w >= T.th2 * dmax2 * (1.0 + 1e-12) && !guard) {
+            cls = 2;
+            const int l = L - 31 + __clz(int(g));
+            two = ((2u * g + 1u) << (l - 1)) - leaf0 < n;
+          } else {
+            cls = 3;
+          }
+        }
+      }
+      uint32_t msk = amask;
+      if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
+      const uint32_t bd = __ballot_sync(kFull, cls == 1);
+      if (cls == 1) {
+        const int pos = nd + __popc(bd & lt);
+        S.drec[pos] = r;
+        S.dmsk[pos] = msk;
+      }
+      nd += __popc(bd);
+      const uint32_t bt = __ballot_sync(kFull, cls == 3);
+      if (cls == 3) S.tstk[nt + __popc(bt & lt)] = make_uint2(g, amask);
+      nt += __popc(bt);
+      const uint32_t b1 = __ballot_sync(kFull, cls == 2);
+      const uint32_t b2 = __ballot_sync(kFull, cls == 2 && two);
+      if (cls == 2) {
+        const int pos = na + __popc(b1 & lt) + __popc(b2 & lt);
+        S.astk[pos] = 2u * g;
+        if (two) S.astk[pos + 1] = 2u * g + 1u;
+      }
+      na += __popc(b1) + __popc(b2);
+      __syncwarp();
+      if (nd > kCapD - 32) {
+        dense(S, nd, T, a, lane);
+        nd = 0;
+        __syncwarp();
+      }
+    } else {
+      break;
+    }
+  }
+  if (nd > 0) dense(S, nd, T, a, lane);
+  store_result(P, k, active, a, lane);
 }
 
 }  // namespace
 
 void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
-  (void)variant;
   const int64_t nt = p.t_end - p.t_begin;
   if (nt <= 0) return;
   const int64_t warps = (nt + 31) / 32;
-  const unsigned grid = unsigned((warps + kWarpsPerBlock - 1) / kWarpsPerBlock);
-  k_force_maskstack<<<grid, 32 * kWarpsPerBlock, 0, s>>>(p);
+  if (variant == 1) {
+    const unsigned grid = unsigned((warps + kV1Warps - 1) / kV1Warps);
+    k_force_maskstack<<<grid, 32 * kV1Warps, 0, s>>>(p);
+  } else {
+    const unsigned grid = unsigned((warps + kV0Warps - 1) / kV0Warps);
+    k_force_grouped<<<grid, 32 * kV0Warps, 0, s>>>(p);
+  }
 }
 
 }  // namespace nb

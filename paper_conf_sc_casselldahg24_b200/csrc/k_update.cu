@@ -61,7 +61,17 @@ __global__ __launch_bounds__(256) void k_scatter1(const uint32_t* __restrict__ s
   out[__float_as_int(vi[i].w)] = src[i];
 }
 
+__global__ __launch_bounds__(256) void k_fill2(float2* __restrict__ p, int64_t count, float2 v) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i < count) p[i] = v;
+}
+
 }  // namespace
+
+void launch_fill_float2(float2* p, int64_t count, float2 v, cudaStream_t s) {
+  if (count <= 0) return;
+  k_fill2<<<unsigned((count + 255) / 256), 256, 0, s>>>(p, count, v);
+}
 
 void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
                      float4* vi_out, cudaStream_t s) {
