@@ -136,6 +136,38 @@ nbody_status nbody_get_state(nbody_ctx *ctx, float *pos_m, float *vel_id);
 
 nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
 
+/* ---- multi-GPU: Hilbert-range partition ------------------
+ * Every rank holds the whole body state and builds the same tree (all stages
+ * up to the tree are deterministic, so the replicas are bit-identical); rank
+ * r computes forces and updates only for the sorted slots
+ * [r*S, min(N, (r+1)*S)), S = ceil(N / world) rounded up to a multiple of 32
+ * [A21].  With a communicator attached, nbody_step ends each step with an
+ * NCCL all-gather of the owned body records (the exchange step), so after
+ * every step all ranks hold the full updated state; results are
+ * bit-identical to one GPU.  nbody_get_accel / nbody_get_interactions are
+ * then collective (every rank must call them).  Without a communicator
+ * (nbody_set_partition) the context computes its slice only and the caller
+ * exchanges slices (nbody_copy_owned) -- the single-GPU emulation the tests
+ * use; by-id getters then write only the owned bodies. */
+
+/* The owned slot range of `rank` for n bodies on `world` ranks (host-only,
+ * no device needed). */
+nbody_status nbody_partition(int64_t n, int rank, int world, int64_t *begin, int64_t *end);
+/* 1 if the library was built with NCCL. */
+int nbody_has_nccl(void);
+/* Write a 128-byte ncclUniqueId (rank 0 creates it, the caller broadcasts it). */
+nbody_status nbody_nccl_unique_id(void *out128);
+/* Create an NCCL communicator for (rank, world) on the current device and
+ * partition the context accordingly.  Collective; call before stepping. */
+nbody_status nbody_attach_nccl(nbody_ctx *ctx, const void *unique_id128, int rank, int world);
+/* Partition without a communicator (1 <= world <= 256). */
+nbody_status nbody_set_partition(nbody_ctx *ctx, int rank, int world);
+/* The context's rank, world and owned sorted-slot range [begin, end). */
+nbody_status nbody_get_partition(nbody_ctx *ctx, int *rank, int *world, int64_t *begin, int64_t *end);
+/* Copy src's owned slice of the body state into dst (same device, same N and
+ * world): the exchange step of an emulated partition. */
+nbody_status nbody_copy_owned(nbody_ctx *dst, nbody_ctx *src);
+
 /* ---- debug views of the last force pass (parity tests) ---------------- */
 /* Hilbert keys of the bodies in the slot order BEFORE the last sort:
  * keys[n] as uint64 (3b bits, Skilling's index). */

@@ -60,6 +60,14 @@ SIGNATURES = {
     "nbody_get_interactions": (_S, [_P, _P]),
     "nbody_get_state": (_S, [_P, _P, _P]),
     "nbody_get_stats": (_S, [_P, C.POINTER(nbody_stats)]),
+    "nbody_partition": (_S, [_I64, C.c_int, C.c_int, C.POINTER(_I64), C.POINTER(_I64)]),
+    "nbody_has_nccl": (C.c_int, []),
+    "nbody_nccl_unique_id": (_S, [_P]),
+    "nbody_attach_nccl": (_S, [_P, _P, C.c_int, C.c_int]),
+    "nbody_set_partition": (_S, [_P, C.c_int, C.c_int]),
+    "nbody_get_partition": (_S, [_P, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(_I64),
+                                 C.POINTER(_I64)]),
+    "nbody_copy_owned": (_S, [_P, _P]),
     "nbody_debug_keys": (_S, [_P, _P]),
     "nbody_debug_perm": (_S, [_P, _P]),
     "nbody_debug_level": (_S, [_P, C.c_int, C.POINTER(_I64), _P, _P, _P]),

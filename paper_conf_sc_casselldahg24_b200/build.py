@@ -41,11 +41,27 @@ def stale() -> bool:
     return any(os.path.getmtime(p) > t for p in _deps())
 
 
+def nccl_dir():
+    """The NCCL the torch wheel ships (nvidia/nccl/{include,lib}), or None."""
+    for p in sys.path:
+        d = os.path.join(p, "nvidia", "nccl")
+        if os.path.exists(os.path.join(d, "include", "nccl.h")) and os.path.isdir(os.path.join(d, "lib")):
+            return d
+    return None
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
+    nccl = []
+    d = nccl_dir()
+    if d:
+        lib = os.path.join(d, "lib")
+        so = sorted(f for f in os.listdir(lib) if f.startswith("libnccl.so"))
+        nccl = ["-DNBODY_WITH_NCCL", "-I", os.path.join(d, "include"), "-L", lib, f"-l:{so[0]}",
+                "-Xlinker", f"-rpath,{lib}"]
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-I", os.path.join(ROOT, "include"), "-o", LIB + ".tmp", *sources()]
+           "-I", os.path.join(ROOT, "include"), *nccl, "-o", LIB + ".tmp", *sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)

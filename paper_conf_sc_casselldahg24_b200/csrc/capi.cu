@@ -4,6 +4,7 @@
 // all on the context stream, captured once into a CUDA graph and replayed.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -12,6 +13,10 @@
 
 #include "../../include/nbody.h"
 #include "internal.cuh"
+
+#ifdef NBODY_WITH_NCCL
+#include <nccl.h>
+#endif
 
 using namespace nb;
 
@@ -48,6 +53,8 @@ struct nbody_ctx {
   float4* acc = nullptr;
   uint32_t* cnt = nullptr;
   float4* stage = nullptr;
+  uint32_t* stage2 = nullptr;
+  float* out3 = nullptr;
   float* bbox_part = nullptr;
   int nbbox = 0;
   GridInfo* grid = nullptr;
@@ -60,6 +67,14 @@ struct nbody_ctx {
 
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t gexec = nullptr;
+
+  // partition over ranks [A21]: rank r owns sorted slots [own_b, own_e),
+  // own_s = slice length (a multiple of 32 so warp groups match 1 GPU)
+  int rank = 0, world = 1;
+  int64_t own_s = 0, own_b = 0, own_e = 0;
+#ifdef NBODY_WITH_NCCL
+  ncclComm_t comm = nullptr;
+#endif
 };
 
 namespace {
@@ -114,6 +129,22 @@ int resolve_bits(int64_t n, int opt) {
 
 size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
 
+constexpr int kMaxWorld = 256;
+constexpr int64_t kPartPad = 32 * kMaxWorld;  // G * S - N < 32 G
+
+// [A21] S = ceil(N / G) rounded up to a multiple of 32 (warp groups then
+// coincide with the single-GPU run, so results are bit-identical).
+void set_part(nbody_ctx* c, int rank, int world) {
+  const int64_t n = c->n;
+  int64_t s = (n + world - 1) / world;
+  s = (s + 31) / 32 * 32;
+  c->rank = rank;
+  c->world = world;
+  c->own_s = s;
+  c->own_b = std::min(n, int64_t(rank) * s);
+  c->own_e = std::min(n, int64_t(rank + 1) * s);
+}
+
 // Tree plan (sizes follow from N alone).  Heap numbering: node
 // (l, j) has global id g = 2^(L-l) + j, so the root is 1, the children of g
 // are 2g and 2g+1 and leaf i is 2^L + i; level l only uses its first
@@ -140,8 +171,8 @@ nbody_status allocate(nbody_ctx* c) {
   const int64_t tiles = sort_tiles(n);
   size_t sz[32];
   int k = 0;
-  sz[k++] = 16 * size_t(n);                         // pm0
-  sz[k++] = 16 * size_t(n);                         // vi0
+  sz[k++] = 16 * size_t(n + kPartPad);              // pm0 (room for G * S records)
+  sz[k++] = 16 * size_t(n + kPartPad);              // vi0
   sz[k++] = 16 * size_t(n);                         // vi1
   sz[k++] = 8 * size_t(n);                          // keys0
   sz[k++] = 8 * size_t(n);                          // keys1
@@ -150,7 +181,9 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 8 * size_t(n);                          // keys_dbg
   sz[k++] = 16 * size_t(n);                         // acc
   sz[k++] = 4 * size_t(n);                          // cnt
-  sz[k++] = 16 * size_t(n);                         // stage
+  sz[k++] = 16 * size_t(n + kPartPad);              // stage (gathered acc for G > 1)
+  sz[k++] = 4 * size_t(n + kPartPad);               // stage2 (gathered counts)
+  sz[k++] = 12 * size_t(n);                         // out3 (by-id outputs for host callers)
   sz[k++] = sizeof(float) * 6 * size_t(c->nbbox);   // bbox partials
   sz[k++] = sizeof(GridInfo);
   sz[k++] = 8;                                      // total
@@ -184,6 +217,8 @@ nbody_status allocate(nbody_ctx* c) {
   c->acc = (float4*)take();
   c->cnt = (uint32_t*)take();
   c->stage = (float4*)take();
+  c->stage2 = (uint32_t*)take();
+  c->out3 = (float*)take();
   c->bbox_part = (float*)take();
   c->grid = (GridInfo*)take();
   c->total = (unsigned long long*)take();
@@ -243,12 +278,14 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   launch_build(c->tree, c->pm[1], s);
   CK(cudaMemsetAsync(c->total, 0, sizeof(unsigned long long), s));
   CK(mark(3));
+  // S6/S7 only on the owned sorted slots [own_b, own_e) [A21]
+  const int64_t ob = c->own_b, oe = c->own_e;
   ForceParams fp;
   fp.t = c->tree;
   fp.leaves = c->pm[1];
   fp.grid = c->grid;
-  fp.t_begin = 0;
-  fp.t_end = n;
+  fp.t_begin = ob;
+  fp.t_end = oe;
   fp.th2 = c->theta * c->theta;
   fp.eps2 = float(c->eps * c->eps);
   fp.acc = c->acc;
@@ -257,7 +294,20 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   launch_force(fp, c->traversal, s);
   CK(mark(4));
   if (integrate) {
-    launch_leapfrog(c->pm[1], c->vi[1], c->acc, n, float(c->dt), c->pm[0], c->vi[0], s);
+    launch_leapfrog(c->pm[1] + ob, c->vi[1] + ob, c->acc, oe - ob, float(c->dt), c->pm[0] + ob, c->vi[0] + ob, s);
+#ifdef NBODY_WITH_NCCL
+    if (c->comm) {  // S0 of the next step: every rank gets every owned slice
+      const size_t cnt = 4 * size_t(c->own_s);
+      ncclResult_t r = ncclGroupStart();
+      if (r == ncclSuccess)
+        r = ncclAllGather(c->pm[0] + int64_t(c->rank) * c->own_s, c->pm[0], cnt, ncclFloat, c->comm, s);
+      if (r == ncclSuccess)
+        r = ncclAllGather(c->vi[0] + int64_t(c->rank) * c->own_s, c->vi[0], cnt, ncclFloat, c->comm, s);
+      const ncclResult_t r2 = ncclGroupEnd();
+      if (r != ncclSuccess || r2 != ncclSuccess)
+        return fail(c, NBODY_ENCCL, ncclGetErrorString(r != ncclSuccess ? r : r2));
+    }
+#endif
   } else {
     CK(cudaMemcpyAsync(c->pm[0], c->pm[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
     CK(cudaMemcpyAsync(c->vi[0], c->vi[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
@@ -322,6 +372,7 @@ nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_
   c->stream = c->own_stream;
   nbody_status s = allocate(c);
   if (s != NBODY_OK) return bail(s);
+  set_part(c, 0, 1);
   c->b = resolve_bits(n, c->key_bits_opt);
   c->key_bytes = 3 * c->b <= 32 ? 4 : 8;
   c->sort.key_bytes = c->key_bytes;
@@ -438,37 +489,53 @@ nbody_status nbody_sync(nbody_ctx* c) {
   return sync_stream(c);
 }
 
-static nbody_status get_by_id3(nbody_ctx* c, const float4* src, float* out) {
+// out[id][3] <- src[i].xyz for the slots [b, e) (src[i] belongs to slot b + i).
+// A host `out` goes through the device staging buffer out3.
+static nbody_status get_by_id3(nbody_ctx* c, const float4* src, int64_t b, int64_t e, float* out) {
   if (!out) return fail(c, NBODY_EINVAL, "null output");
   const int64_t n = c->n;
-  if (is_device_ptr(out)) {
-    launch_scatter_by_id3(src, c->vi[0], n, out, c->stream);
-    CK(cudaGetLastError());
-    return sync_stream(c);
-  }
-  float* tmp = reinterpret_cast<float*>(c->stage);
-  launch_scatter_by_id3(src, c->vi[0], n, tmp, c->stream);
+  const bool dev = is_device_ptr(out);
+  float* dst = dev ? out : c->out3;
+  if (!dev && (b > 0 || e < n)) CK(cudaMemcpyAsync(dst, out, 12 * size_t(n), cudaMemcpyDefault, c->stream));
+  launch_scatter_by_id3(src, c->vi[0] + b, e - b, dst, c->stream);
   CK(cudaGetLastError());
-  CK(cudaMemcpyAsync(out, tmp, 12 * size_t(n), cudaMemcpyDefault, c->stream));
+  if (!dev) CK(cudaMemcpyAsync(out, dst, 12 * size_t(n), cudaMemcpyDefault, c->stream));
   return sync_stream(c);
 }
+
+#ifdef NBODY_WITH_NCCL
+// Collective: gather every rank's owned slice of src (S records of `words`
+// 4-byte words) into dst, indexed by slot.
+static nbody_status gather_owned(nbody_ctx* c, const void* src, void* dst, size_t words) {
+  const ncclResult_t r = ncclAllGather(src, dst, words * size_t(c->own_s), ncclFloat, c->comm, c->stream);
+  if (r != ncclSuccess) return fail(c, NBODY_ENCCL, ncclGetErrorString(r));
+  return NBODY_OK;
+}
+#endif
 
 nbody_status nbody_get_accel(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
-  return get_by_id3(c, c->acc, out);
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) {
+    nbody_status s = gather_owned(c, c->acc, c->stage, 4);
+    if (s != NBODY_OK) return s;
+    return get_by_id3(c, c->stage, 0, c->n, out);
+  }
+#endif
+  return get_by_id3(c, c->acc, c->own_b, c->own_e, out);
 }
 
 nbody_status nbody_get_positions(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
-  return get_by_id3(c, c->pm[0], out);
+  return get_by_id3(c, c->pm[0], 0, c->n, out);
 }
 
 nbody_status nbody_get_velocities(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
-  return get_by_id3(c, c->vi[0], out);
+  return get_by_id3(c, c->vi[0], 0, c->n, out);
 }
 
 nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
@@ -476,16 +543,110 @@ nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
   if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
   if (!out) return fail(c, NBODY_EINVAL, "null output");
   const int64_t n = c->n;
-  if (is_device_ptr(out)) {
-    launch_scatter_by_id1(c->cnt, c->vi[0], n, out, c->stream);
-    CK(cudaGetLastError());
-    return sync_stream(c);
+  const uint32_t* src = c->cnt;
+  int64_t b = c->own_b, e = c->own_e;
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) {
+    nbody_status s = gather_owned(c, c->cnt, c->stage2, 1);
+    if (s != NBODY_OK) return s;
+    src = c->stage2;
+    b = 0;
+    e = n;
   }
-  uint32_t* tmp = reinterpret_cast<uint32_t*>(c->stage);
-  launch_scatter_by_id1(c->cnt, c->vi[0], n, tmp, c->stream);
+#endif
+  const bool dev = is_device_ptr(out);
+  uint32_t* dst = dev ? out : reinterpret_cast<uint32_t*>(c->out3);
+  if (!dev && (b > 0 || e < n)) CK(cudaMemcpyAsync(dst, out, 4 * size_t(n), cudaMemcpyDefault, c->stream));
+  launch_scatter_by_id1(src, c->vi[0] + b, e - b, dst, c->stream);
   CK(cudaGetLastError());
-  CK(cudaMemcpyAsync(out, tmp, 4 * size_t(n), cudaMemcpyDefault, c->stream));
+  if (!dev) CK(cudaMemcpyAsync(out, dst, 4 * size_t(n), cudaMemcpyDefault, c->stream));
   return sync_stream(c);
+}
+
+// ---- partition / multi-GPU -------------------------------------------------
+
+nbody_status nbody_set_partition(nbody_ctx* c, int rank, int world) {
+  CHECK_CTX(c);
+  if (world < 1 || world > kMaxWorld || rank < 0 || rank >= world)
+    return fail(c, NBODY_EINVAL, "need 0 <= rank < world <= 256");
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is attached");
+#endif
+  set_part(c, rank, world);
+  drop_graph(c);
+  return NBODY_OK;
+}
+
+nbody_status nbody_get_partition(nbody_ctx* c, int* rank, int* world, int64_t* begin, int64_t* end) {
+  CHECK_CTX(c);
+  if (rank) *rank = c->rank;
+  if (world) *world = c->world;
+  if (begin) *begin = c->own_b;
+  if (end) *end = c->own_e;
+  return NBODY_OK;
+}
+
+nbody_status nbody_copy_owned(nbody_ctx* dst, nbody_ctx* src) {
+  CHECK_CTX(dst);
+  nbody_ctx* c = dst;
+  if (!src || src->n != dst->n || src->world != dst->world) return fail(c, NBODY_EINVAL, "incompatible contexts");
+  const int64_t b = src->own_b, len = src->own_e - src->own_b;
+  if (len <= 0) return NBODY_OK;
+  CK(cudaStreamSynchronize(src->stream));
+  CK(cudaMemcpyAsync(dst->pm[0] + b, src->pm[0] + b, 16 * size_t(len), cudaMemcpyDeviceToDevice, dst->stream));
+  CK(cudaMemcpyAsync(dst->vi[0] + b, src->vi[0] + b, 16 * size_t(len), cudaMemcpyDeviceToDevice, dst->stream));
+  return sync_stream(dst);
+}
+
+nbody_status nbody_partition(int64_t n, int rank, int world, int64_t* begin, int64_t* end) {
+  if (n < 1 || world < 1 || world > kMaxWorld || rank < 0 || rank >= world || !begin || !end) return NBODY_EINVAL;
+  nbody_ctx tmp;
+  tmp.n = n;
+  set_part(&tmp, rank, world);
+  *begin = tmp.own_b;
+  *end = tmp.own_e;
+  return NBODY_OK;
+}
+
+int nbody_has_nccl(void) {
+#ifdef NBODY_WITH_NCCL
+  return 1;
+#else
+  return 0;
+#endif
+}
+
+nbody_status nbody_nccl_unique_id(void* out) {
+  if (!out) return NBODY_EINVAL;
+#ifdef NBODY_WITH_NCCL
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return NBODY_ENCCL;
+  std::memcpy(out, &id, sizeof(id));
+  return NBODY_OK;
+#else
+  return NBODY_ENCCL;
+#endif
+}
+
+nbody_status nbody_attach_nccl(nbody_ctx* c, const void* unique_id, int rank, int world) {
+  CHECK_CTX(c);
+  if (!unique_id || world < 1 || world > kMaxWorld || rank < 0 || rank >= world)
+    return fail(c, NBODY_EINVAL, "need a unique id and 0 <= rank < world <= 256");
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is already attached");
+  ncclUniqueId id;
+  std::memcpy(&id, unique_id, sizeof(id));
+  const ncclResult_t r = ncclCommInitRank(&c->comm, world, id, rank);
+  if (r != ncclSuccess) {
+    c->comm = nullptr;
+    return fail(c, NBODY_ENCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+  }
+  set_part(c, rank, world);
+  drop_graph(c);
+  return NBODY_OK;
+#else
+  return fail(c, NBODY_ENCCL, "library built without NCCL");
+#endif
 }
 
 nbody_status nbody_get_state(nbody_ctx* c, float* pos_m, float* vel_id) {
@@ -592,6 +753,9 @@ void nbody_destroy(nbody_ctx* c) {
   if (!c) return;
   if (c->stream) cudaStreamSynchronize(c->stream);
   drop_graph(c);
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) ncclCommDestroy(c->comm);
+#endif
   if (c->arena) cudaFree(c->arena);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);

@@ -128,6 +128,29 @@ class NBody:
         self._ck(self.lib.nbody_get_stats(self.h, C.byref(s)))
         return {f: getattr(s, f) for f, _ in s._fields_}
 
+    # -- multi-GPU ---------------------------------------------------------
+    def set_partition(self, rank: int, world: int):
+        self._ck(self.lib.nbody_set_partition(self.h, int(rank), int(world)))
+
+    def partition(self):
+        r, w = C.c_int(), C.c_int()
+        b, e = C.c_int64(), C.c_int64()
+        self._ck(self.lib.nbody_get_partition(self.h, C.byref(r), C.byref(w), C.byref(b), C.byref(e)))
+        return r.value, w.value, b.value, e.value
+
+    def copy_owned_from(self, other: "NBody"):
+        self._ck(self.lib.nbody_copy_owned(self.h, other.h))
+
+    def attach_nccl(self, unique_id: bytes, rank: int, world: int):
+        buf = C.create_string_buffer(bytes(unique_id), 128)
+        self._ck(self.lib.nbody_attach_nccl(self.h, buf, int(rank), int(world)))
+
+    def attach_process_group(self, rank: int, world: int, group=None):
+        """Bootstrap the library's NCCL communicator through torch.distributed:
+        rank 0 creates the unique id, the process group broadcasts it."""
+        from .dist import broadcast_unique_id
+        self.attach_nccl(broadcast_unique_id(rank, group), rank, world)
+
     # -- debug views (parity tests) -----------------------------------------
     def debug_keys(self):
         out = np.empty(self.n, np.uint64)
