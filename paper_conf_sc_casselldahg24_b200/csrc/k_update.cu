@@ -85,10 +85,12 @@ void launch_pack_bodies(const float* pos, const float* vel, const float* mass, i
 }
 
 void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s) {
+  if (n <= 0) return;  // a rank may own no slots
   k_scatter3<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
 }
 
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s) {
+  if (n <= 0) return;
   k_scatter1<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
 }
 
