@@ -60,8 +60,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
         so = sorted(f for f in os.listdir(lib) if f.startswith("libnccl.so"))
         nccl = ["-DNBODY_WITH_NCCL", "-I", os.path.join(d, "include"), "-L", lib, f"-l:{so[0]}",
                 "-Xlinker", f"-rpath,{lib}"]
+    extra = os.environ.get("NBODY_NVCC_FLAGS", "").split()  # tuning experiments only
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-I", os.path.join(ROOT, "include"), *nccl, "-o", LIB + ".tmp", *sources()]
+           "-I", os.path.join(ROOT, "include"), *nccl, *extra, "-o", LIB + ".tmp", *sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)

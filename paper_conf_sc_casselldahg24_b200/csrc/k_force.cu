@@ -18,19 +18,25 @@
 // thresholds on the squared distance, pred[g] the exact fp64 (com, s^2) of
 // an internal node.
 //
-// Variant 0 (default), group-classified walk.  A warp owns 32
+// Variant 0 (default), group-classified transposed walk.  A warp owns 32
 // Hilbert-consecutive targets with bounding box B.
-//   A. Lanes classify 32 tree nodes at a time against B with exact fp64
-//      bounds of the opening test over all of B: SURE_ACCEPT (every lane
-//      accepts: the node joins the warp's common list), SURE_REJECT (every
-//      lane opens it: its children are classified next) or MIXED.  Leaves
-//      reached here are common too.  Every node reaching A has been opened
-//      by every lane, so common entries are in every lane's list.
-//   B. The common list is evaluated densely: each entry is read once from
-//      shared memory (broadcast) and every lane interacts with it.
-//   C. Each MIXED node is walked with the per-lane mask stack below,
-//      starting with all lanes.
-// Variant 1, the mask-stack walk from the root for every warp.
+//   A. Box phase (lanes = nodes): lanes classify 32 nodes at a time against B
+//      with exact fp64 bounds of the opening test over all of B: every lane
+//      accepts (-> dense list, all lanes), every lane opens (-> children are
+//      box-classified next) or mixed (-> T with all lanes in the mask).
+//      Every node reaching A has been opened by every lane, so this is exact.
+//   T. Transposed phase (lanes = nodes, loop over targets): each lane takes a
+//      (node, mask of the targets that reached it) entry and evaluates the
+//      per-target opening test for all 32 targets, whose positions are
+//      broadcast from shared memory -- one warp instruction decides 32
+//      node-target pairs.  Accepting targets -> a dense entry (record, mask);
+//      opening targets -> both children enter T with that mask.  Leaves carry
+//      thresholds (-inf, -inf): always accepted, except by the target itself.
+//   D. Dense phase (lanes = targets): each entry is read once from shared
+//      memory (broadcast) and every lane in its mask interacts with it; full-
+//      mask and partial-mask entries are kept in separate lists.
+// Variant 1, the mask-stack walk from the root for every warp (the simpler
+// exact design, kept as a cross-check and as the overflow path of T).
 //
 // Mask stack: a warp-uniform DFS stack of (sibling pair, mask of the lanes
 // that reached it), held in registers (lane i holds entry i; depth <= L+1 <
@@ -246,18 +252,36 @@ __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForcePa
   store_result(P, k, active, a, lane);
 }
 
+
 // ------------------------------------------------------------ variant 0 ----
 constexpr int kV0Warps = 4;
-constexpr int kCapA = 256;  // box-phase stack (ids)
-constexpr int kCapT = 512;  // transposed-phase stack (id, mask)
-constexpr int kCapD = 128;  // dense list (record, mask)
+// Sized for 8 blocks x 4 warps per SM (26.4 KB shared memory per block);
+// stack overflow is handled (box phase: hand over as MIXED; transposed
+// phase: per-lane mask walk), so the capacities only affect speed.
+#ifndef NBODY_CAP_T
+#define NBODY_CAP_T 352
+#endif
+#ifndef NBODY_V0_MINB
+#define NBODY_V0_MINB 8
+#endif
+constexpr int kCapA = 128;          // box-phase stack (ids)
+constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
+#ifndef NBODY_CAP_F
+#define NBODY_CAP_F 96
+#endif
+#ifndef NBODY_CAP_P
+#define NBODY_CAP_P 64
+#endif
+constexpr int kCapF = NBODY_CAP_F;  // dense list: entries every active lane interacts with
+constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 
 struct V0Smem {
-  float4 tgt[32];       // the warp's target positions
-  float4 drec[kCapD];   // dense list: monopole / body record
-  uint32_t dmsk[kCapD]; //             lanes that interact with it
+  float4 tgt[32];        // the warp's target positions
+  float4 frec[kCapF];    // monopole / body records, all lanes
+  float4 prec[kCapP];    // monopole / body records, ...
+  uint32_t pmsk[kCapP];  // ... for the lanes in the mask
   uint32_t astk[kCapA];
-  uint2 tstk[kCapT];    // (id, mask of the targets that reached it)
+  uint2 tstk[kCapT];     // (id, mask of the targets that reached it)
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -271,19 +295,42 @@ __device__ __forceinline__ float warp_maxf(float v) {
   return v;
 }
 
-// Dense list: entry e interacts with the lanes in dmsk[e].
-__device__ __forceinline__ void dense(const V0Smem& S, int nd, const Target& T, Acc& a, int lane) {
+// a += m r / (|r|^2 + eps^2)^(3/2), r = s - x.  kSoft (eps > 0): r2 > 0 always.
+template <bool kSoft>
+__device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const Target& T) {
+  const float dx = s.x - T.x, dy = s.y - T.y, dz = s.z - T.z;
+  const float r2 = fmaf(dz, dz, fmaf(dy, dy, fmaf(dx, dx, T.eps2)));
+  float inv = rsqrt_fast(r2);
+  if (!kSoft) inv = r2 > 0.f ? inv : 0.f;
+  const float w = m * inv * inv * inv;
+  a.x = fmaf(w, dx, a.x);
+  a.y = fmaf(w, dy, a.y);
+  a.z = fmaf(w, dz, a.z);
+}
+
+template <bool kSoft>
+__device__ __forceinline__ void dense_full(const V0Smem& S, int nf, const Target& T, Acc& a) {
 #pragma unroll 4
-  for (int e = 0; e < nd; ++e) {
-    const float4 s = S.drec[e];
-    const bool on = (S.dmsk[e] >> lane) & 1u;
-    const Probe p = probe(s, T);
-    a.add(on, p.dx, p.dy, p.dz, p.d2, s.w, T.eps2);
+  for (int e = 0; e < nf; ++e) {
+    const float4 s = S.frec[e];
+    interact<kSoft>(a, s, s.w, T);
+  }
+  a.n += uint32_t(nf);
+}
+
+template <bool kSoft>
+__device__ __forceinline__ void dense_part(const V0Smem& S, int np, const Target& T, Acc& a, int lane) {
+#pragma unroll 4
+  for (int e = 0; e < np; ++e) {
+    const float4 s = S.prec[e];
+    const bool on = (S.pmsk[e] >> lane) & 1u;
+    interact<kSoft>(a, s, on ? s.w : 0.f, T);
     a.n += on;
   }
 }
 
-__global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForceParams P) {
+template <bool kSoft>
+__global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(const ForceParams P) {
   __shared__ V0Smem s_all[kV0Warps];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   V0Smem& S = s_all[w];
@@ -309,9 +356,38 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
   const double bly = warp_minf(active ? T.y : inf), bhy = warp_maxf(active ? T.y : -inf);
   const double blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
 
-  int na = 1, nt = 0, nd = 0;
+  int na = 1, nt = 0, nf = 0, np = 0;
   if (lane == 0) S.astk[0] = 1u;
   __syncwarp();
+
+  // Append (record r, lane mask msk) to the dense lists: full when every
+  // active lane interacts with it.
+  auto append = [&](bool want, const float4& r, uint32_t msk) {
+    const bool full = want && msk == amask;
+    const bool part = want && msk != amask;
+    const uint32_t bf = __ballot_sync(kFull, full);
+    const uint32_t bp = __ballot_sync(kFull, part);
+    if (full) S.frec[nf + __popc(bf & lt)] = r;
+    if (part) {
+      const int pos = np + __popc(bp & lt);
+      S.prec[pos] = r;
+      S.pmsk[pos] = msk;
+    }
+    nf += __popc(bf);
+    np += __popc(bp);
+  };
+  auto flush = [&](bool all) {
+    __syncwarp();
+    if (nf > kCapF - 32 || (all && nf > 0)) {
+      dense_full<kSoft>(S, nf, T, a);
+      nf = 0;
+    }
+    if (np > kCapP - 32 || (all && np > 0)) {
+      dense_part<kSoft>(S, np, T, a, lane);
+      np = 0;
+    }
+    __syncwarp();
+  };
 
   while (true) {
     if (nt >= 32 || (na == 0 && nt > 0)) {
@@ -349,14 +425,7 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
         }
       }
       if (g >= leaf0 && g - kid0 < 32u) am &= ~(1u << (g - kid0));  // a leaf never acts on itself
-      // dense-list append
-      const uint32_t bd = __ballot_sync(kFull, am != 0u);
-      if (am) {
-        const int pos = nd + __popc(bd & lt);
-        S.drec[pos] = r;
-        S.dmsk[pos] = am;
-      }
-      nd += __popc(bd);
+      append(am != 0u, r, am);
       // children of opened nodes, with the mask of the targets that opened them
       const int l = L - 31 + __clz(int(g));
       const bool two = rm && (((2u * g + 1u) << (l - 1)) - leaf0) < n;
@@ -370,12 +439,7 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
         if (two) S.tstk[pos + 1] = make_uint2(2u * g + 1u, rm);
       }
       nt += __popc(b1) + __popc(b2);
-      __syncwarp();
-      if (nd > kCapD - 32) {
-        dense(S, nd, T, a, lane);
-        nd = 0;
-        __syncwarp();
-      }
+      flush(false);
       // no room (never observed at the sizes we run): walk those subtrees per lane
       uint32_t spill = __ballot_sync(kFull, rm != 0u && !room);
       while (spill) {
@@ -384,7 +448,6 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
         const uint32_t gs = __shfl_sync(kFull, g, src);
         const uint32_t ms = __shfl_sync(kFull, rm, src);
         mask_walk(W, T, kid, a, lane, 2u * gs, ms);
-        // (the walk starts at the left child; the right child, if any:)
         const int ls = L - 31 + __clz(int(gs));
         if ((((2u * gs + 1u) << (ls - 1)) - leaf0) < n) mask_walk(W, T, kid, a, lane, 2u * gs + 1u, ms);
       }
@@ -397,7 +460,7 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
       __syncwarp();
       na = base;
       const bool guard = na + 64 > kCapA;
-      int cls = 0;  // 1 dense (all lanes), 2 expand, 3 transposed
+      int cls = 0;  // 1 dense, 2 expand, 3 transposed
       float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
       bool two = false;
       if (has) {
@@ -430,13 +493,7 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
       }
       uint32_t msk = amask;
       if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
-      const uint32_t bd = __ballot_sync(kFull, cls == 1);
-      if (cls == 1) {
-        const int pos = nd + __popc(bd & lt);
-        S.drec[pos] = r;
-        S.dmsk[pos] = msk;
-      }
-      nd += __popc(bd);
+      append(cls == 1, r, msk);
       const uint32_t bt = __ballot_sync(kFull, cls == 3);
       if (cls == 3) S.tstk[nt + __popc(bt & lt)] = make_uint2(g, amask);
       nt += __popc(bt);
@@ -448,17 +505,12 @@ __global__ __launch_bounds__(32 * kV0Warps) void k_force_grouped(const ForcePara
         if (two) S.astk[pos + 1] = 2u * g + 1u;
       }
       na += __popc(b1) + __popc(b2);
-      __syncwarp();
-      if (nd > kCapD - 32) {
-        dense(S, nd, T, a, lane);
-        nd = 0;
-        __syncwarp();
-      }
+      flush(false);
     } else {
       break;
     }
   }
-  if (nd > 0) dense(S, nd, T, a, lane);
+  flush(true);
   store_result(P, k, active, a, lane);
 }
 
@@ -473,7 +525,10 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
     k_force_maskstack<<<grid, 32 * kV1Warps, 0, s>>>(p);
   } else {
     const unsigned grid = unsigned((warps + kV0Warps - 1) / kV0Warps);
-    k_force_grouped<<<grid, 32 * kV0Warps, 0, s>>>(p);
+    if (p.eps2 > 0.f)
+      k_force_grouped<true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    else
+      k_force_grouped<false><<<grid, 32 * kV0Warps, 0, s>>>(p);
   }
 }
 
