@@ -264,10 +264,13 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   CK(mark(0));
   launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
   launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
+  CK(cudaMemsetAsync(c->sort.ghist, 0, sizeof(uint32_t) * 8 * 256, s));
+  c->sort.hist_ready = true;  // the key kernel fills the sort's digit histograms
   if (c->key_bytes == 4)
-    launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), s);
+    launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), c->sort.ghist, c->sort.passes, s);
   else
-    launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), s);
+    launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), c->sort.ghist,
+                  c->sort.passes, s);
   if (debug) {
     CK(cudaMemcpyAsync(c->keys_dbg, c->keys[0], size_t(c->key_bytes) * n, cudaMemcpyDeviceToDevice, s));
   }
@@ -314,8 +317,8 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   }
   CK(mark(5));
   c->ev_valid = tm;
-  // K1 2 + K2 1 + K3 (1 + passes) + K4 1 + K5 L + K6 1 + K7 1
-  c->kernels_per_step = 2 + 1 + 1 + c->sort.passes + 1 + c->tree.L + 1 + (integrate ? 1 : 0);
+  // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 L + K6 1 + K7 1
+  c->kernels_per_step = 2 + 1 + c->sort.passes + 1 + c->tree.L + 1 + (integrate ? 1 : 0);
   CK(cudaGetLastError());
   return NBODY_OK;
 }

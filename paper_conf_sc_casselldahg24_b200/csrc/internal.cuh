@@ -61,8 +61,11 @@ struct ForceParams {
 // ---- K1 / K2 --------------------------------------------------------------
 void launch_bbox_partial(const float4* pm, int64_t n, float* partial, int nblocks, cudaStream_t s);
 void launch_bbox_final(const float* partial, int nparts, int b, GridInfo* g, cudaStream_t s);
-void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, cudaStream_t s);
-void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, cudaStream_t s);
+// keys + the sort's digit histograms (ghist[passes][256], must be zeroed)
+void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, uint32_t* ghist, int passes,
+                   cudaStream_t s);
+void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
+                   int passes, cudaStream_t s);
 
 // ---- K3 radix sort ---------------------------------------------------------
 struct SortPlan {
@@ -73,6 +76,7 @@ struct SortPlan {
   uint32_t* ghist;    // [8][256]
   uint32_t* status;   // [passes][tiles][256]
   uint32_t* tile_ctr; // [8]
+  bool hist_ready;    // ghist already filled (by the key kernel)
 };
 int64_t sort_tiles(int64_t n);
 size_t sort_scratch_bytes(int64_t n);

@@ -123,20 +123,52 @@ __device__ __forceinline__ unsigned long long hilbert3(uint32_t x0, uint32_t x1,
   return (spread3(x0) << 2) | (spread3(x1) << 1) | spread3(x2);
 }
 
+constexpr int kKeysThreads = 256;
+
+// Keys, plus the radix-sort digit histograms of every pass (the onesweep
+// sort's upfront histogram, fused here so the keys are read only by the
+// sort passes).  Grid-stride; per-block shared histograms; a warp whose 32
+// keys share a digit adds it once (common for the high digits: the input is
+// the previous step's Hilbert order).
 template <class K>
-__global__ __launch_bounds__(256) void k_keys(const float4* __restrict__ pm, int64_t n, const GridInfo* __restrict__ gi,
-                                              K* __restrict__ keys) {
-  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (i >= n) return;
+__global__ __launch_bounds__(kKeysThreads) void k_keys(const float4* __restrict__ pm, int64_t n,
+                                                       const GridInfo* __restrict__ gi, K* __restrict__ keys,
+                                                       uint32_t* __restrict__ ghist, int passes) {
+  __shared__ uint32_t sh[8 * 256];
+  for (int i = threadIdx.x; i < passes * 256; i += kKeysThreads) sh[i] = 0;
+  __syncthreads();
   const GridInfo g = *gi;
-  const float4 p = __ldg(pm + i);
   const uint32_t qmax = (1u << g.b) - 1u;
-  // q_k = min(2^b - 1, floor((x_k - lo_k) * inv)) in fp64; the operand is
-  // >= 0, so truncation is the floor.
-  const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), double(g.lo[0])), g.inv)));
-  const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), double(g.lo[1])), g.inv)));
-  const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), double(g.lo[2])), g.inv)));
-  keys[i] = K(hilbert3(q0, q1, q2, g.b));
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = int64_t(gridDim.x) * kKeysThreads;
+  for (int64_t base = int64_t(blockIdx.x) * kKeysThreads + (threadIdx.x & ~31); base < n; base += stride) {
+    const int64_t i = base + lane;
+    const bool ok = i < n;
+    K key = 0;
+    if (ok) {
+      const float4 p = __ldg(pm + i);
+      // q_k = min(2^b - 1, floor((x_k - lo_k) * inv)) in fp64; the operand is
+      // >= 0, so truncation is the floor.
+      const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), double(g.lo[0])), g.inv)));
+      const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), double(g.lo[1])), g.inv)));
+      const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), double(g.lo[2])), g.inv)));
+      key = K(hilbert3(q0, q1, q2, g.b));
+      keys[i] = key;
+    }
+    const uint32_t act = __ballot_sync(0xffffffffu, ok);
+    for (int ps = 0; ps < passes; ++ps) {
+      const uint32_t d = uint32_t(key >> (8 * ps)) & 255u;
+      const uint32_t d0 = __shfl_sync(0xffffffffu, d, 0);
+      if (__all_sync(0xffffffffu, !ok || d == d0)) {
+        if (lane == 0) atomicAdd(&sh[ps * 256 + d0], uint32_t(__popc(act)));
+      } else if (ok) {
+        atomicAdd(&sh[ps * 256 + d], 1u);
+      }
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < passes * 256; i += kKeysThreads)
+    if (sh[i]) atomicAdd(&ghist[i], sh[i]);
 }
 
 }  // namespace
@@ -149,12 +181,20 @@ void launch_bbox_final(const float* partial, int nparts, int b, GridInfo* g, cud
   k_bbox_final<<<1, 32, 0, s>>>(partial, nparts, b, g);
 }
 
-void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, cudaStream_t s) {
-  k_keys<uint32_t><<<unsigned((n + 255) / 256), 256, 0, s>>>(pm, n, g, keys);
+static unsigned keys_grid(int64_t n) {
+  const int64_t want = (n + kKeysThreads - 1) / kKeysThreads;
+  const int64_t cap = 8 * kNumSMs;  // enough blocks to saturate HBM, few global histogram flushes
+  return unsigned(want < cap ? want : cap);
 }
 
-void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, cudaStream_t s) {
-  k_keys<unsigned long long><<<unsigned((n + 255) / 256), 256, 0, s>>>(pm, n, g, keys);
+void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, uint32_t* ghist, int passes,
+                   cudaStream_t s) {
+  k_keys<uint32_t><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
+}
+
+void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
+                   int passes, cudaStream_t s) {
+  k_keys<unsigned long long><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
 }
 
 }  // namespace nb

@@ -80,7 +80,7 @@ __device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t* s_tmp) {
 }
 
 template <class K, bool kFirst, bool kWriteKeys>
-__global__ __launch_bounds__(kThreads) void k_onesweep(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+__global__ __launch_bounds__(kThreads, 2) void k_onesweep(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                        K* __restrict__ kout, uint32_t* __restrict__ vout, int64_t n,
                                                        int shift, const uint32_t* __restrict__ ghist,
                                                        uint32_t* __restrict__ status, uint32_t* __restrict__ tile_ctr) {
@@ -200,11 +200,13 @@ void run_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s
     set_attr<K, false, true>(); set_attr<K, false, false>();
     attrs = true;
   }
-  cudaMemsetAsync(p.ghist, 0, sizeof(uint32_t) * 8 * kRadix, s);
   cudaMemsetAsync(p.tile_ctr, 0, sizeof(uint32_t) * 8, s);
   cudaMemsetAsync(p.status, 0, sizeof(uint32_t) * size_t(p.passes) * size_t(p.tiles) * kRadix, s);
-  const int hb = int(p.tiles < 4 * kNumSMs ? p.tiles : int64_t(4 * kNumSMs));
-  k_hist<K><<<hb, kThreads, 0, s>>>(static_cast<const K*>(keys[0]), p.n, p.passes, p.ghist);
+  if (!p.hist_ready) {
+    cudaMemsetAsync(p.ghist, 0, sizeof(uint32_t) * 8 * kRadix, s);
+    const int hb = int(p.tiles < 4 * kNumSMs ? p.tiles : int64_t(4 * kNumSMs));
+    k_hist<K><<<hb, kThreads, 0, s>>>(static_cast<const K*>(keys[0]), p.n, p.passes, p.ghist);
+  }
   for (int pass = 0; pass < p.passes; ++pass) {
     const int in = pass & 1, out = in ^ 1;
     const K* kin = static_cast<const K*>(keys[in]);
