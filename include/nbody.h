@@ -136,6 +136,14 @@ nbody_status nbody_get_state(nbody_ctx *ctx, float *pos_m, float *vel_id);
 
 nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
 
+/* ---- NEXT-1: the paper's All-Pairs baseline, sampled -----------
+ * Exact softened direct sum of Eq. 1 [A1] at the current positions,
+ * fp64 arithmetic and accumulation, for the bodies with ids[nt] (host or
+ * device; host ids are range-checked); out[nt][3] fp64, host or device.
+ * Deterministic (fixed-order reduction).  Used to measure Barnes-Hut
+ * accuracy against the exact field (config 5). */
+nbody_status nbody_direct_accel(nbody_ctx *ctx, const int64_t *ids, int64_t nt, double *out);
+
 /* ---- multi-GPU: Hilbert-range partition ------------------
  * Every rank holds the whole body state and builds the same tree (all stages
  * up to the tree are deterministic, so the replicas are bit-identical); rank

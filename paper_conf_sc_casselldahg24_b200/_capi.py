@@ -60,6 +60,7 @@ SIGNATURES = {
     "nbody_get_interactions": (_S, [_P, _P]),
     "nbody_get_state": (_S, [_P, _P, _P]),
     "nbody_get_stats": (_S, [_P, C.POINTER(nbody_stats)]),
+    "nbody_direct_accel": (_S, [_P, _P, _I64, _P]),
     "nbody_partition": (_S, [_I64, C.c_int, C.c_int, C.POINTER(_I64), C.POINTER(_I64)]),
     "nbody_has_nccl": (C.c_int, []),
     "nbody_nccl_unique_id": (_S, [_P]),

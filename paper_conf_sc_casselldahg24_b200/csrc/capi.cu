@@ -566,6 +566,38 @@ nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
   return sync_stream(c);
 }
 
+// ---- NEXT-1: all-pairs reference ------------------------------------------
+
+nbody_status nbody_direct_accel(nbody_ctx* c, const int64_t* ids, int64_t nt, double* out) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (nt < 0 || (nt > 0 && (!ids || !out))) return fail(c, NBODY_EINVAL, "bad target list");
+  if (nt == 0) return NBODY_OK;
+  const bool ids_dev = is_device_ptr(ids);
+  if (!ids_dev)
+    for (int64_t i = 0; i < nt; ++i)
+      if (ids[i] < 0 || ids[i] >= c->n) return fail(c, NBODY_EINVAL, "id out of range");
+  const int64_t chunks = direct_chunks(c->n, nt);
+  cudaStream_t s = c->stream;
+  char* tmp = nullptr;
+  const size_t bi = align_up(8 * size_t(nt)), bt = align_up(4 * size_t(nt)), bp = align_up(32 * size_t(chunks * nt));
+  const size_t bo = align_up(24 * size_t(nt));
+  CK(cudaMallocAsync(reinterpret_cast<void**>(&tmp), bi + bt + bp + bo, s));
+  int64_t* d_ids = reinterpret_cast<int64_t*>(tmp);
+  uint32_t* d_tslot = reinterpret_cast<uint32_t*>(tmp + bi);
+  double4* d_part = reinterpret_cast<double4*>(tmp + bi + bt);
+  double* d_out = reinterpret_cast<double*>(tmp + bi + bt + bp);
+  cudaError_t e = cudaMemcpyAsync(d_ids, ids, 8 * size_t(nt), cudaMemcpyDefault, s);
+  if (e == cudaSuccess) {
+    launch_direct(c->pm[0], c->vi[0], c->n, d_ids, nt, c->eps * c->eps, c->stage2, d_tslot, d_part, d_out, s);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(out, d_out, 24 * size_t(nt), cudaMemcpyDefault, s);
+  cudaFreeAsync(tmp, s);
+  if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
+  return sync_stream(c);
+}
+
 // ---- partition / multi-GPU -------------------------------------------------
 
 nbody_status nbody_set_partition(nbody_ctx* c, int rank, int world) {

@@ -92,6 +92,11 @@ void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 
+// ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
+int64_t direct_chunks(int64_t n, int64_t nt);
+void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t* ids, int64_t nt, double eps2,
+                   uint32_t* slot_of, uint32_t* tslot, double4* part, double* out, cudaStream_t s);
+
 // ---- K7 and helpers --------------------------------------------------------
 void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
                      float4* vi_out, cudaStream_t s);

@@ -128,6 +128,13 @@ class NBody:
         self._ck(self.lib.nbody_get_stats(self.h, C.byref(s)))
         return {f: getattr(s, f) for f, _ in s._fields_}
 
+    def direct_accel(self, ids):
+        """Exact fp64 direct-sum accelerations (NEXT-1) for the given body ids."""
+        ids = np.ascontiguousarray(ids, np.int64)
+        out = np.empty((len(ids), 3), np.float64)
+        self._ck(self.lib.nbody_direct_accel(self.h, _ptr(ids), len(ids), _ptr(out)))
+        return out
+
     # -- multi-GPU ---------------------------------------------------------
     def set_partition(self, rank: int, world: int):
         self._ck(self.lib.nbody_set_partition(self.h, int(rank), int(world)))
