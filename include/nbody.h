@@ -71,7 +71,12 @@ enum {
   /* 1 = record CUDA events around each stage of a pass issued by
    * nbody_compute_accel / nbody_step with graphs off; nbody_get_stats then
    * reports the device time of each stage of the last pass.  Default 0. */
-  NBODY_OPT_TIMING = 5
+  NBODY_OPT_TIMING = 5,
+  /* BUILDTREEACCUMULATEMASS kernel variant: 0 = fused 1024-leaf subtrees
+   * in shared memory + one block for the top levels (default), 1 = one
+   * kernel per level (the paper's level-by-level parallel-for).  Both
+   * produce bit-identical records. */
+  NBODY_OPT_BUILD = 6
 };
 
 typedef struct {

@@ -28,6 +28,7 @@ struct nbody_ctx {
   int key_bytes = 8;
   bool use_graph = true;
   int traversal = 0;
+  int build_variant = 0;  // 0 fused subtrees, 1 level by level
   bool timing = false;
   cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
   bool ev_valid = false;
@@ -278,7 +279,14 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   c->perm_buf = launch_radix_sort(c->sort, c->keys, c->idx, s);
   CK(mark(2));
   launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
-  launch_build(c->tree, c->pm[1], s);
+  int build_kernels;
+  if (c->build_variant == 1) {
+    launch_build(c->tree, c->pm[1], s);
+    build_kernels = c->tree.L;
+  } else {
+    launch_build_fused(c->tree, c->pm[1], debug, s);
+    build_kernels = c->tree.L < 1 ? 0 : (c->tree.L > 10 ? 2 : 1);
+  }
   CK(cudaMemsetAsync(c->total, 0, sizeof(unsigned long long), s));
   CK(mark(3));
   // S6/S7 only on the owned sorted slots [own_b, own_e) [A21]
@@ -318,7 +326,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   CK(mark(5));
   c->ev_valid = tm;
   // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 L + K6 1 + K7 1
-  c->kernels_per_step = 2 + 1 + c->sort.passes + 1 + c->tree.L + 1 + (integrate ? 1 : 0);
+  c->kernels_per_step = 2 + 1 + c->sort.passes + 1 + build_kernels + 1 + (integrate ? 1 : 0);
   CK(cudaGetLastError());
   return NBODY_OK;
 }
@@ -402,6 +410,11 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
     case NBODY_OPT_USE_GRAPH:
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "use_graph must be 0 or 1");
       c->use_graph = value != 0;
+      return NBODY_OK;
+    case NBODY_OPT_BUILD:
+      if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown build variant");
+      c->build_variant = int(value);
+      drop_graph(c);
       return NBODY_OK;
     case NBODY_OPT_TIMING:
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "timing must be 0 or 1");

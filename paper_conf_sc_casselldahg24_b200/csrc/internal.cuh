@@ -87,7 +87,10 @@ int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaSt
 // ---- K4 / K5 ---------------------------------------------------------------
 void launch_permute(const float4* pm_in, const float4* vi_in, const uint32_t* perm, int64_t n, float4* pm_out,
                     float4* vi_out, cudaStream_t s);
-void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);
+void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);  // level by level (reference)
+// levels 1..10 fused per 1024-leaf subtree + one block for the top levels;
+// keep_all also stores every node's moments/box (debug views)
+void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, cudaStream_t s);
 
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);

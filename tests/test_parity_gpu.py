@@ -266,3 +266,21 @@ def test_direct_accel_at_10M_sampled(NB, oracle):
     sim.compute_accel()
     bh = sim.get_accel()[ids]
     assert np.median(rel_errors(bh, got)) < 1e-2
+
+
+@pytest.mark.parametrize("n", [1000, 1025, 70_001, 2_000_003])
+def test_build_variants_bit_identical(NB, n):
+    """Fused-subtree build == level-by-level build, every level."""
+    pos, vel, mass = generate("clustered", n, 70)
+    sims = []
+    for variant in (0, 1):
+        s = NB(n, 0.5, EPS, DT)
+        s.set_option(6, variant)  # NBODY_OPT_BUILD
+        s.set_bodies(pos, vel, mass)
+        s.compute_accel()
+        sims.append(s)
+    L = sims[0].stats()["levels"]
+    for l in range(1, L + 1):
+        for a, b in zip(sims[0].debug_level(l), sims[1].debug_level(l)):
+            assert (a == b).all(), l
+    assert (sims[0].get_accel() == sims[1].get_accel()).all()
