@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--n", type=int, default=0, help="override N (testing only)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target oracle force-sample time")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle force-sample time")
     return ap.parse_args()
 
 
@@ -155,8 +155,14 @@ def cpu_oracle_sample(pos, vel, mass, cfg, target_seconds, seed=0):
     r.tree.force(cfg["theta"], cfg["eps"], probe)
     t_probe = time.perf_counter() - tf0
     t_prep = max(0.0, t_all - t_probe)
+    # size the sample from a second, larger probe (thread start-up dominates a small one)
     per_target = max(t_probe / len(probe), 1e-9)
-    ns = int(min(n, max(len(probe), target_seconds / per_target)))
+    ns = int(min(n, max(len(probe), 0.15 * target_seconds / per_target)))
+    targets = np.sort(rng.choice(n, ns, replace=False))
+    tf0 = time.perf_counter()
+    r.tree.force(cfg["theta"], cfg["eps"], targets)
+    per_target = max((time.perf_counter() - tf0) / ns, 1e-9)
+    ns = int(min(n, max(ns, target_seconds / per_target)))
     targets = np.sort(rng.choice(n, ns, replace=False))
     tf0 = time.perf_counter()
     _, cnt = r.tree.force(cfg["theta"], cfg["eps"], targets)

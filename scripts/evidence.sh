@@ -8,5 +8,5 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --c
   python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1; echo launches=$?
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_force -s 1 -c 1 -o gpurun_out/force_${tag} \
   python scripts/run_pass.py --passes 2 > /dev/null 2>&1; echo ncu_force=$?
-timeout 900 ncu --set full --clock-control none -k regex:"k_onesweep|k_hist|k_build|k_permute|k_keys|k_bbox|k_leapfrog" -s 40 -c 40 -o gpurun_out/build_${tag} \
+timeout 900 ncu --set full --clock-control none -k regex:"k_onesweep|k_build|k_permute|k_keys|k_bbox|k_leapfrog" -s 13 -c 13 -o gpurun_out/build_${tag} \
   python scripts/run_pass.py --passes 3 > /dev/null 2>&1; echo ncu_build=$?
