@@ -352,9 +352,9 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
 
   // group box over the active lanes (exact fp32 min/max, used in fp64)
   const float inf = __int_as_float(0x7f800000);
-  const double blx = warp_minf(active ? T.x : inf), bhx = warp_maxf(active ? T.x : -inf);
-  const double bly = warp_minf(active ? T.y : inf), bhy = warp_maxf(active ? T.y : -inf);
-  const double blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
+  const float blx = warp_minf(active ? T.x : inf), bhx = warp_maxf(active ? T.x : -inf);
+  const float bly = warp_minf(active ? T.y : inf), bhy = warp_maxf(active ? T.y : -inf);
+  const float blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
 
   int na = 1, nt = 0, nf = 0, np = 0;
   if (lane == 0) S.astk[0] = 1u;
@@ -468,21 +468,26 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
           cls = 1;
           r = __ldg(W.rec + g);
         } else {
-          const double4 p = W.pred[g];
-          // exact bounds of |com - x|^2 over the box
-          const double ax0 = __dsub_rn(blx, p.x), ax1 = __dsub_rn(p.x, bhx);
-          const double ay0 = __dsub_rn(bly, p.y), ay1 = __dsub_rn(p.y, bhy);
-          const double az0 = __dsub_rn(blz, p.z), az1 = __dsub_rn(p.z, bhz);
-          const double nx = fmax(0.0, fmax(ax0, ax1)), ny = fmax(0.0, fmax(ay0, ay1)),
-                       nz = fmax(0.0, fmax(az0, az1));
-          const double fx = fmax(fabs(ax0), fabs(ax1)), fy = fmax(fabs(ay0), fabs(ay1)),
-                       fz = fmax(fabs(az0), fabs(az1));
-          const double dmin2 = nx * nx + ny * ny + nz * nz;
-          const double dmax2 = fx * fx + fy * fy + fz * fz;
-          if (p.w < T.th2 * dmin2 * (1.0 - 1e-12)) {
+          // fp32 bounds of |c32 - x|^2 over the box against the node's filter
+          // thresholds.  Both the box bound and every target's filter value
+          // are fp32 evaluations from the same c32, equal to the exact
+          // |c32 - x|^2 within 5u each, so Dmin2 (1 - 4e-6) > hi => every
+          // target's d2 > hi => all accept; Dmax2 (1 + 4e-6) < lo => all open
+          // (DESIGN.md "fp32 filter").
+          r = __ldg(W.rec + g);
+          const float2 c = __ldg(W.rc + g);
+          const float ax0 = blx - r.x, ax1 = r.x - bhx;
+          const float ay0 = bly - r.y, ay1 = r.y - bhy;
+          const float az0 = blz - r.z, az1 = r.z - bhz;
+          const float nx = fmaxf(0.f, fmaxf(ax0, ax1)), ny = fmaxf(0.f, fmaxf(ay0, ay1)),
+                      nz = fmaxf(0.f, fmaxf(az0, az1));
+          const float fx = fmaxf(fabsf(ax0), fabsf(ax1)), fy = fmaxf(fabsf(ay0), fabsf(ay1)),
+                      fz = fmaxf(fabsf(az0), fabsf(az1));
+          const float dmin2 = fmaf(nz, nz, fmaf(ny, ny, nx * nx));
+          const float dmax2 = fmaf(fz, fz, fmaf(fy, fy, fx * fx));
+          if (dmin2 * (1.f - 4e-6f) > c.y) {
             cls = 1;
-            r = __ldg(W.rec + g);
-          } else if (p.w >= T.th2 * dmax2 * (1.0 + 1e-12) && !guard) {
+          } else if (dmax2 * (1.f + 4e-6f) < c.x && !guard) {
             cls = 2;
             const int l = L - 31 + __clz(int(g));
             two = ((2u * g + 1u) << (l - 1)) - leaf0 < n;
