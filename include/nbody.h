@@ -76,7 +76,13 @@ enum {
    * in shared memory + one block for the top levels (default), 1 = one
    * kernel per level (the paper's level-by-level parallel-for).  Both
    * produce bit-identical records. */
-  NBODY_OPT_BUILD = 6
+  NBODY_OPT_BUILD = 6,
+  /* Tree reuse (NEXT-3(iii); Iwasawa et al., cited at P:320) [A23]: k >= 1;
+   * nbody_step re-sorts on steps 0, k, 2k, ... after nbody_set_bodies and
+   * otherwise keeps the previous Hilbert order, rebuilding the BVH bottom-up
+   * over it at the current positions (no keys, no sort, no permutation).
+   * Default 1 (the paper's Alg. 6: sort every step). */
+  NBODY_OPT_SORT_EVERY = 7
 };
 
 typedef struct {

@@ -230,13 +230,18 @@ class StepResult:
 
 
 def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_bits: int = 16,
-         integrate: bool = True, targets=None, nthreads: int = 0) -> StepResult:
+         integrate: bool = True, targets=None, nthreads: int = 0, resort: bool = True) -> StepResult:
     """One step of Alg. 6 on fp32 state in the current slot order.
 
     O8 [A14] kick-drift leapfrog, v_{+1/2} = v_{-1/2} + a dt, x += v_{+1/2} dt,
     evaluated in fp64 and stored in fp32 (the state precision of the path).
     With ``targets`` (sorted slots) only those bodies get forces and the
     update is skipped.
+
+    ``resort=False`` is the tree-reuse variant (NEXT-3(iii), Iwasawa et al.
+    as cited at P:320, [A23]): HILBERTSORT is skipped and the bodies keep
+    their current slot order (the previous step's Hilbert order); the BVH is
+    rebuilt bottom-up over that order at the current positions.
     """
     t0 = time.perf_counter()
     pos = _f32(pos, (-1, 3))
@@ -244,9 +249,13 @@ def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_b
     mass = _f32(mass, (-1,))
     n = len(pos)
     ids = np.arange(n, dtype=np.int64) if ids is None else np.asarray(ids, np.int64)
-    b = resolve_key_bits(n, key_bits)
-    k = keys(pos, b)                           # O1-O3
-    perm = sort_perm(k)                        # O4
+    if resort:
+        b = resolve_key_bits(n, key_bits)
+        k = keys(pos, b)                       # O1-O3
+        perm = sort_perm(k)                    # O4
+    else:
+        k = np.zeros(0, np.uint64)
+        perm = np.arange(n, dtype=np.uint32)
     ps, vs, ms, ids_s = pos[perm], vel[perm], mass[perm], ids[perm]  # O5 [A11]
     tree = Tree(ps, ms)                        # O6
     full = targets is None

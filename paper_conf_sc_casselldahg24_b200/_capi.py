@@ -24,6 +24,7 @@ NBODY_OPT_USE_GRAPH = 3
 NBODY_OPT_TRAVERSAL = 4
 NBODY_OPT_TIMING = 5
 NBODY_OPT_BUILD = 6
+NBODY_OPT_SORT_EVERY = 7
 
 _STATUS = {0: "NBODY_OK", -1: "NBODY_EINVAL", -2: "NBODY_ENOMEM", -3: "NBODY_ECUDA", -4: "NBODY_ENCCL",
            -5: "NBODY_ESTATE"}

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -68,6 +69,10 @@ struct nbody_ctx {
 
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t gexec = nullptr;
+  cudaGraph_t graph_reuse = nullptr;    // tree-reuse step (NEXT-3(iii))
+  cudaGraphExec_t gexec_reuse = nullptr;
+  int sort_every = 1;                   // re-sort every k-th step
+  bool last_sorted = false;
 
   // partition over ranks [A21]: rank r owns sorted slots [own_b, own_e),
   // own_s = slice length (a multiple of 32 so warp groups match 1 GPU)
@@ -251,34 +256,50 @@ nbody_status allocate(nbody_ctx* c) {
 void drop_graph(nbody_ctx* c) {
   if (c->gexec) cudaGraphExecDestroy(c->gexec);
   if (c->graph) cudaGraphDestroy(c->graph);
+  if (c->gexec_reuse) cudaGraphExecDestroy(c->gexec_reuse);
+  if (c->graph_reuse) cudaGraphDestroy(c->graph_reuse);
   c->gexec = nullptr;
   c->graph = nullptr;
+  c->gexec_reuse = nullptr;
+  c->graph_reuse = nullptr;
 }
 
 // One force pass (and optionally the update) on stream s.  State enters in
 // (pm[0], vi[0]) in the current slot order and leaves there in the new
 // Hilbert order.
-nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool debug) {
+nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool debug, bool resort = true) {
   const int64_t n = c->n;
   const bool tm = c->timing && s == c->stream;
   auto mark = [&](int i) -> cudaError_t { return tm ? cudaEventRecord(c->ev[i], s) : cudaSuccess; };
   CK(mark(0));
   launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
   launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
-  CK(cudaMemsetAsync(c->sort.ghist, 0, sizeof(uint32_t) * 8 * 256, s));
-  c->sort.hist_ready = true;  // the key kernel fills the sort's digit histograms
-  if (c->key_bytes == 4)
-    launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), c->sort.ghist, c->sort.passes, s);
-  else
-    launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), c->sort.ghist,
-                  c->sort.passes, s);
-  if (debug) {
-    CK(cudaMemcpyAsync(c->keys_dbg, c->keys[0], size_t(c->key_bytes) * n, cudaMemcpyDeviceToDevice, s));
+  int front_kernels = 2;
+  if (resort) {
+    CK(cudaMemsetAsync(c->sort.ghist, 0, sizeof(uint32_t) * 8 * 256, s));
+    c->sort.hist_ready = true;  // the key kernel fills the sort's digit histograms
+    if (c->key_bytes == 4)
+      launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), c->sort.ghist, c->sort.passes, s);
+    else
+      launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), c->sort.ghist,
+                    c->sort.passes, s);
+    if (debug) {
+      CK(cudaMemcpyAsync(c->keys_dbg, c->keys[0], size_t(c->key_bytes) * n, cudaMemcpyDeviceToDevice, s));
+    }
+    CK(mark(1));
+    c->perm_buf = launch_radix_sort(c->sort, c->keys, c->idx, s);
+    CK(mark(2));
+    launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
+    front_kernels += 1 + c->sort.passes + 1;
+  } else {
+    // tree reuse (NEXT-3(iii), [A23]): keep the current (previous Hilbert)
+    // order; the leaves are the current state
+    CK(mark(1));
+    CK(mark(2));
+    CK(cudaMemcpyAsync(c->pm[1], c->pm[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(c->vi[1], c->vi[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
   }
-  CK(mark(1));
-  c->perm_buf = launch_radix_sort(c->sort, c->keys, c->idx, s);
-  CK(mark(2));
-  launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
+  c->last_sorted = resort;
   int build_kernels;
   if (c->build_variant == 1) {
     launch_build(c->tree, c->pm[1], s);
@@ -325,16 +346,18 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   }
   CK(mark(5));
   c->ev_valid = tm;
-  // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 L + K6 1 + K7 1
-  c->kernels_per_step = 2 + 1 + c->sort.passes + 1 + build_kernels + 1 + (integrate ? 1 : 0);
+  // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 + K6 1 + K7 1
+  c->kernels_per_step = front_kernels + build_kernels + 1 + (integrate ? 1 : 0);
   CK(cudaGetLastError());
   return NBODY_OK;
 }
 
-nbody_status build_graph(nbody_ctx* c) {
-  drop_graph(c);
+// Capture one full step (resort = sorting step, else tree-reuse step).
+nbody_status build_graph(nbody_ctx* c, bool resort) {
+  cudaGraph_t& graph = resort ? c->graph : c->graph_reuse;
+  cudaGraphExec_t& exec = resort ? c->gexec : c->gexec_reuse;
   CK(cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal));
-  nbody_status st = enqueue_pass(c, c->cap_stream, true, false);
+  nbody_status st = enqueue_pass(c, c->cap_stream, true, false, resort);
   cudaGraph_t g = nullptr;
   cudaError_t e = cudaStreamEndCapture(c->cap_stream, &g);
   if (st != NBODY_OK) {
@@ -342,8 +365,8 @@ nbody_status build_graph(nbody_ctx* c) {
     return st;
   }
   if (e != cudaSuccess) return fail(c, NBODY_ECUDA, std::string("graph capture: ") + cudaGetErrorString(e));
-  c->graph = g;
-  CK(cudaGraphInstantiate(&c->gexec, g, 0));
+  graph = g;
+  CK(cudaGraphInstantiate(&exec, g, 0));
   return NBODY_OK;
 }
 
@@ -416,6 +439,10 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       c->build_variant = int(value);
       drop_graph(c);
       return NBODY_OK;
+    case NBODY_OPT_SORT_EVERY:
+      if (value < 1 || value > (int64_t(1) << 30)) return fail(c, NBODY_EINVAL, "sort_every must be >= 1");
+      c->sort_every = int(value);
+      return NBODY_OK;
     case NBODY_OPT_TIMING:
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "timing must be 0 or 1");
       c->timing = value != 0;
@@ -481,18 +508,22 @@ nbody_status nbody_step(nbody_ctx* c, int nsteps) {
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
   if (nsteps < 0) return fail(c, NBODY_EINVAL, "nsteps < 0");
   if (nsteps == 0) return NBODY_OK;
-  if (c->use_graph) {
-    if (!c->gexec) {
-      nbody_status s = build_graph(c);
+  for (int i = 0; i < nsteps; ++i) {
+    // step k of this body set re-sorts iff k % sort_every == 0 (always the first)
+    const bool resort = (c->steps + i) % c->sort_every == 0;
+    if (c->use_graph) {
+      cudaGraphExec_t& exec = resort ? c->gexec : c->gexec_reuse;
+      if (!exec) {
+        nbody_status s = build_graph(c, resort);
+        if (s != NBODY_OK) return s;
+      }
+      CK(cudaGraphLaunch(exec, c->stream));
+      c->ev_valid = false;
+    } else {
+      nbody_status s = enqueue_pass(c, c->stream, true, false, resort);
       if (s != NBODY_OK) return s;
     }
-    for (int i = 0; i < nsteps; ++i) CK(cudaGraphLaunch(c->gexec, c->stream));
-    c->ev_valid = false;
-  } else {
-    for (int i = 0; i < nsteps; ++i) {
-      nbody_status s = enqueue_pass(c, c->stream, true, false);
-      if (s != NBODY_OK) return s;
-    }
+    c->last_sorted = resort;
   }
   c->have_force = true;
   c->keys_dbg_valid = false;
@@ -770,6 +801,7 @@ nbody_status nbody_debug_perm(nbody_ctx* c, uint32_t* perm) {
   CHECK_CTX(c);
   if (!perm) return fail(c, NBODY_EINVAL, "null output");
   if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  if (!c->last_sorted) return fail(c, NBODY_ESTATE, "the last pass reused the tree order (no sort)");
   CK(cudaMemcpyAsync(perm, c->idx[c->perm_buf], 4 * size_t(c->n), cudaMemcpyDefault, c->stream));
   return sync_stream(c);
 }

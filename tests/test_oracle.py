@@ -418,3 +418,31 @@ def test_leapfrog_conserves_momentum_with_exact_forces(oracle):
     p1 = (m[:, None].astype(float) * u.astype(float)).sum(axis=0)
     scale = (mass[:, None] * np.abs(vel)).sum()
     assert np.abs(p1 - p0).max() / scale < 1e-6
+
+
+# ------------------------------------------------- NEXT-3(iii) tree reuse ---
+def test_tree_reuse_on_sorted_state_equals_resort(oracle):
+    """resort=False on bodies already in Hilbert order (the previous step's
+    output, positions unchanged) is the same step as a fresh sort."""
+    pos, vel, mass = generate("plummer", 3000, 81)
+    r0 = oracle.step(pos, vel, mass, theta=0.5, eps=1e-3, dt=0.0)
+    a = oracle.step(r0.pos, r0.vel, r0.mass, r0.ids, theta=0.5, eps=1e-3, dt=1e-3)
+    b = oracle.step(r0.pos, r0.vel, r0.mass, r0.ids, theta=0.5, eps=1e-3, dt=1e-3, resort=False)
+    assert (a.perm == np.arange(3000)).all()
+    assert (a.acc == b.acc).all() and (a.count == b.count).all() and (a.pos == b.pos).all()
+
+
+def test_tree_reuse_keeps_exactness_properties(oracle):
+    """Any leaf order gives a valid BVH: theta = 0 is still the direct sum and
+    every list still partitions the other bodies."""
+    pos, vel, mass = generate("uniform", 700, 82)  # unsorted array order
+    r = oracle.step(pos, vel, mass, theta=0.0, eps=1e-3, dt=1e-3, integrate=False, resort=False)
+    assert (r.ids == np.arange(700)).all()
+    d = oracle.direct(pos, mass, 1e-3)
+    assert _rel_err(r.acc, d).max() <= 1e-12 and (r.count == 699).all()
+    r = oracle.step(pos, vel, mass, theta=0.5, eps=1e-3, dt=1e-3, integrate=False, resort=False)
+    for k in (0, 350, 699):
+        cover = np.zeros(700, np.int64)
+        for l, j in r.tree.force_list(0.5, 1e-3, k):
+            cover[j << l: min((j + 1) << l, 700)] += 1
+        assert cover[k] == 0 and (np.delete(cover, k) == 1).all()
