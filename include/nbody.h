@@ -102,6 +102,11 @@ typedef struct {
 /* Library version (major*10000 + minor*100 + patch). */
 int nbody_version(void);
 
+/* Make `device` the calling thread's current CUDA device for this library
+ * (the library links its own CUDA runtime; callers that select devices
+ * through another runtime, e.g. PyTorch, call this before nbody_create). */
+nbody_status nbody_select_device(int device);
+
 /* Create a context for n bodies on the current CUDA device.
  *   n in [1, 2^30 - 1] (the sort packs counts in 30 bits); theta >= 0 (opening parameter, accept a node iff
  *   s^2 < theta^2 d^2, [A3]); eps >= 0 (Plummer softening [A1]); dt finite

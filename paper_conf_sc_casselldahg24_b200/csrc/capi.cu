@@ -381,6 +381,16 @@ extern "C" {
 
 int nbody_version(void) { return 100; }
 
+nbody_status nbody_select_device(int device) {
+  int count = 0;
+  if (cudaGetDeviceCount(&count) != cudaSuccess) {
+    cudaGetLastError();
+    return NBODY_ECUDA;
+  }
+  if (device < 0 || device >= count) return NBODY_EINVAL;
+  return cudaSetDevice(device) == cudaSuccess ? NBODY_OK : NBODY_ECUDA;
+}
+
 nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx** out) {
   if (!out) return NBODY_EINVAL;
   *out = nullptr;

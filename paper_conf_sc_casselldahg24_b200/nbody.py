@@ -46,9 +46,20 @@ class NBody:
     """One simulation context: ``NBody(n, theta, eps, dt)``."""
 
     def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
-                 stream=None, use_graph: bool = True, traversal: int = 0):
+                 stream=None, use_graph: bool = True, traversal: int = 0, device=None):
         self.lib = _capi.load()
         self.n = int(n)
+        if device is None:  # follow PyTorch's current device when torch has one
+            try:
+                import torch
+                if torch.cuda.is_available():
+                    device = torch.cuda.current_device()
+            except ImportError:
+                pass
+        if device is not None:
+            st = self.lib.nbody_select_device(int(device))
+            if st != 0:
+                raise _capi.NBodyError(st, f"nbody_select_device({device}) failed")
         h = C.c_void_p()
         st = self.lib.nbody_create(self.n, float(theta), float(eps), float(dt), C.byref(h))
         if st != 0:
