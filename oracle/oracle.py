@@ -62,6 +62,10 @@ def lib():
         L.orc_tree_count.restype = C.c_int64
         L.orc_tree_level.argtypes = [_P, C.c_int, _P, _P, _P, _P, _P]
         L.orc_force.argtypes = [_P, C.c_double, C.c_double, _i64p, C.c_int64, _f64p, _P, C.c_int]
+        L.orc_force_q.argtypes = [_P, C.c_double, C.c_double, C.c_int, _i64p, C.c_int64, _f64p, _P, C.c_int]
+        L.orc_force_q.restype = C.c_int
+        L.orc_tree_level_quad.argtypes = [_P, C.c_int, _f64p]
+        L.orc_tree_level_quad.restype = C.c_int
         L.orc_force_list.argtypes = [_P, C.c_double, C.c_double, C.c_int64, _i64p, C.c_int64]
         L.orc_force_list.restype = C.c_int64
         L.orc_direct.argtypes = [C.c_int64, _f32p, _f32p, C.c_double, _i64p, C.c_int64, _f64p, C.c_int]
@@ -184,14 +188,21 @@ class Tree:
                                  d.lo.ctypes.data, d.hi.ctypes.data), "tree_level")
         return d
 
-    def force(self, theta: float, eps: float, targets=None, nthreads: int = 0):
-        """O7 -- per-target DFS; returns (acc fp64 [nt,3], interactions int64 [nt])."""
+    def force(self, theta: float, eps: float, targets=None, nthreads: int = 0, quad: bool = False):
+        """O7 -- per-target DFS; returns (acc fp64 [nt,3], interactions int64 [nt]).
+        ``quad`` adds the quadrupole of every accepted node (NEXT-4 [A24])."""
         t = np.arange(self.n, dtype=np.int64) if targets is None else np.ascontiguousarray(targets, np.int64)
         acc = np.empty((len(t), 3))
         cnt = np.empty(len(t), np.int64)
-        _ok(lib().orc_force(self._h, float(theta), float(eps), t, len(t), acc, cnt.ctypes.data, int(nthreads)),
-            "force")
+        _ok(lib().orc_force_q(self._h, float(theta), float(eps), int(bool(quad)), t, len(t), acc, cnt.ctypes.data,
+                              int(nthreads)), "force")
         return acc, cnt
+
+    def level_quad(self, l: int):
+        """[A24] second moments about the COM of level l: fp64 [c, 6] (xx, yy, zz, xy, xz, yz)."""
+        out = np.empty((self.count(l), 6))
+        _ok(lib().orc_tree_level_quad(self._h, l, out), "tree_level_quad")
+        return out
 
     def force_list(self, theta: float, eps: float, target: int):
         """O7 interaction list of one target: int64 [len, 2] of (level, index), DFS order."""
@@ -230,7 +241,8 @@ class StepResult:
 
 
 def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_bits: int = 16,
-         integrate: bool = True, targets=None, nthreads: int = 0, resort: bool = True) -> StepResult:
+         integrate: bool = True, targets=None, nthreads: int = 0, resort: bool = True,
+         quad: bool = False) -> StepResult:
     """One step of Alg. 6 on fp32 state in the current slot order.
 
     O8 [A14] kick-drift leapfrog, v_{+1/2} = v_{-1/2} + a dt, x += v_{+1/2} dt,
@@ -260,7 +272,7 @@ def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_b
     tree = Tree(ps, ms)                        # O6
     full = targets is None
     tg = np.arange(n, dtype=np.int64) if full else np.ascontiguousarray(targets, np.int64)
-    acc, cnt = tree.force(theta, eps, tg, nthreads)   # O7
+    acc, cnt = tree.force(theta, eps, tg, nthreads, quad)   # O7 (+ NEXT-4 quadrupoles)
     if integrate and full:                     # O8
         v_new = vs.astype(np.float64) + acc * dt
         x_new = ps.astype(np.float64) + v_new * dt

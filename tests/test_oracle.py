@@ -446,3 +446,74 @@ def test_tree_reuse_keeps_exactness_properties(oracle):
         for l, j in r.tree.force_list(0.5, 1e-3, k):
             cover[j << l: min((j + 1) << l, 700)] += 1
         assert cover[k] == 0 and (np.delete(cover, k) == 1).all()
+
+
+# --------------------------------------------------- NEXT-4 quadrupoles ------
+def test_second_moments_match_brute_force(oracle):
+    """[A24] S = sum m (x - com)(x - com)^T over each node's leaf range."""
+    rng = np.random.default_rng(91)
+    n = 777
+    pos = rng.normal(size=(n, 3)).astype(np.float32)
+    mass = rng.uniform(0.5, 2.0, n).astype(np.float32)
+    t = oracle.Tree(pos, mass)
+    ii, jj = [0, 1, 2, 0, 0, 1], [0, 1, 2, 1, 2, 2]
+    for l in range(0, t.L + 1):
+        S = t.level_quad(l)
+        com = t.level(l).com
+        for j in range(0, t.count(l), max(1, t.count(l) // 25)):
+            a, b = j << l, min((j + 1) << l, n)
+            y = pos[a:b].astype(float) - com[j]
+            m = mass[a:b].astype(float)
+            scale = math.fsum(m * (y ** 2).sum(axis=1)) + 1e-300
+            for q in range(6):
+                ref = math.fsum(m * y[:, ii[q]] * y[:, jj[q]])
+                assert abs(S[j, q] - ref) <= 1e-12 * scale
+
+
+def test_quadrupole_two_point_closed_form(oracle):
+    """Masses m/2 at c -+ (s, 0, 0), target on the axis at distance D: the
+    monopole is off by 3 s^2/D^2, the quadrupole term removes it (what is left
+    is O(s^4/D^4))."""
+    s = 0.25
+    for D in (4.0, 8.0):
+        pos = np.float32([[-s, 0, 0], [s, 0, 0], [D, 0, 0]])  # target last in Hilbert order (cell 2^b-1,0,0)
+        mass = np.float32([0.5, 0.5, 1e-6])
+        exact = 0.5 / (D - s) ** 2 + 0.5 / (D + s) ** 2
+        mono = oracle.step(pos, np.zeros_like(pos), mass, theta=1.0, eps=0.0, dt=0.0, integrate=False)
+        quad = oracle.step(pos, np.zeros_like(pos), mass, theta=1.0, eps=0.0, dt=0.0, integrate=False, quad=True)
+        k = int(np.nonzero(mono.ids == 2)[0][0])
+        assert mono.count[k] == 1  # one accepted node: the pair
+        em = abs(-mono.acc[k, 0] - exact) / exact
+        eq = abs(-quad.acc[k, 0] - exact) / exact
+        assert em == pytest.approx(3 * s * s / D ** 2, rel=0.2)
+        assert eq < 10 * (s / D) ** 4
+
+
+def test_quadrupole_far_cluster_is_third_order(oracle):
+    rng = np.random.default_rng(4)
+    blob = rng.uniform(-0.5, 0.5, (256, 3)) * [1.0, 2.0, 0.5]
+    em, eq = [], []
+    for d in (8.0, 16.0, 32.0):
+        pos = np.vstack([blob, [[d, -1.0, -0.25]]]).astype(np.float32)
+        mass = np.full(len(pos), 1.0 / 256, np.float32)
+        exact = oracle.direct(pos, mass, 0.0, targets=[256])[0]
+        for q, out in ((False, em), (True, eq)):
+            r = oracle.step(pos, np.zeros_like(pos), mass, theta=1.0, eps=0.0, dt=0.0, integrate=False, quad=q)
+            assert r.count[256] == 1
+            out.append(np.linalg.norm(r.acc[256] - exact) / np.linalg.norm(exact))
+    assert all(q < m / 10 for q, m in zip(eq, em))
+    for a, b in zip(eq, eq[1:]):
+        assert 6.0 < a / b < 18.0  # at least third order
+
+
+def test_quadrupole_improves_accuracy_same_lists(oracle):
+    pos, vel, mass = generate("uniform", 4096, 92)
+    m = oracle.step(pos, vel, mass, theta=0.6, eps=1e-3, dt=0.0, integrate=False)
+    q = oracle.step(pos, vel, mass, theta=0.6, eps=1e-3, dt=0.0, integrate=False, quad=True)
+    assert (m.count == q.count).all()  # the opening test does not change
+    exact = oracle.direct(m.tree.pos, m.tree.mass, 1e-3)
+    rm = np.sqrt(np.mean(_rel_err(m.acc, exact) ** 2))
+    rq = np.sqrt(np.mean(_rel_err(q.acc, exact) ** 2))
+    assert rq < 0.5 * rm
+    z = oracle.step(pos, vel, mass, theta=0.0, eps=1e-3, dt=0.0, integrate=False, quad=True)
+    assert _rel_err(z.acc, exact).max() <= 1e-12
