@@ -82,7 +82,14 @@ enum {
    * otherwise keeps the previous Hilbert order, rebuilding the BVH bottom-up
    * over it at the current positions (no keys, no sort, no permutation).
    * Default 1 (the paper's Alg. 6: sort every step). */
-  NBODY_OPT_SORT_EVERY = 7
+  NBODY_OPT_SORT_EVERY = 7,
+  /* Multipole order (NEXT-4; "the algorithms extend to multipoles")
+   * [A24]: 1 = monopole (default, the paper's exposition), 2 = monopole +
+   * quadrupole: every node also carries its second mass moment about the COM
+   * (fp64, parallel-axis theorem) and accepted nodes add the softened
+   * quadrupole term.  The opening test, hence every interaction list, is
+   * unchanged.  Allocates 80 B per internal node on first use. */
+  NBODY_OPT_MULTIPOLE = 8
 };
 
 typedef struct {
@@ -205,6 +212,11 @@ nbody_status nbody_debug_perm(nbody_ctx *ctx, uint32_t *perm);
  * interaction); box[count][6] fp32 = (lo xyz, hi xyz).  Any of pred, rec,
  * box may be NULL; pass all NULL to query *count. */
 nbody_status nbody_debug_level(nbody_ctx *ctx, int level, int64_t *count, double *pred, float *rec, float *box);
+
+/* NEXT-4: second mass moments about the COM of level l in [1, L] after
+ * nbody_compute_accel with NBODY_OPT_MULTIPOLE = 2: S[count][6] fp64 =
+ * (xx, yy, zz, xy, xz, yz) [A24]. */
+nbody_status nbody_debug_quad(nbody_ctx *ctx, int level, double *S);
 
 /* Human-readable description of the last error on this context (never NULL). */
 const char *nbody_last_error(const nbody_ctx *ctx);

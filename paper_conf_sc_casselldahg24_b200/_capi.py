@@ -25,6 +25,7 @@ NBODY_OPT_TRAVERSAL = 4
 NBODY_OPT_TIMING = 5
 NBODY_OPT_BUILD = 6
 NBODY_OPT_SORT_EVERY = 7
+NBODY_OPT_MULTIPOLE = 8
 
 _STATUS = {0: "NBODY_OK", -1: "NBODY_EINVAL", -2: "NBODY_ENOMEM", -3: "NBODY_ECUDA", -4: "NBODY_ENCCL",
            -5: "NBODY_ESTATE"}
@@ -72,6 +73,7 @@ SIGNATURES = {
     "nbody_get_partition": (_S, [_P, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(_I64),
                                  C.POINTER(_I64)]),
     "nbody_copy_owned": (_S, [_P, _P]),
+    "nbody_debug_quad": (_S, [_P, C.c_int, _P]),
     "nbody_debug_keys": (_S, [_P, _P]),
     "nbody_debug_perm": (_S, [_P, _P]),
     "nbody_debug_level": (_S, [_P, C.c_int, C.POINTER(_I64), _P, _P, _P]),

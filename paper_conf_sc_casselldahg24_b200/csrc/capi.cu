@@ -73,6 +73,7 @@ struct nbody_ctx {
   cudaGraphExec_t gexec_reuse = nullptr;
   int sort_every = 1;                   // re-sort every k-th step
   bool last_sorted = false;
+  void* quad_arena = nullptr;           // NEXT-4 S64 + qf (lazy)
 
   // partition over ranks [A21]: rank r owns sorted slots [own_b, own_e),
   // own_s = slice length (a multiple of 32 so warp groups match 1 GPU)
@@ -301,7 +302,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   }
   c->last_sorted = resort;
   int build_kernels;
-  if (c->build_variant == 1) {
+  if (c->build_variant == 1 && !c->tree.quad) {  // the level-by-level variant is monopole only
     launch_build(c->tree, c->pm[1], s);
     build_kernels = c->tree.L;
   } else {
@@ -447,6 +448,22 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
     case NBODY_OPT_BUILD:
       if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown build variant");
       c->build_variant = int(value);
+      drop_graph(c);
+      return NBODY_OK;
+    case NBODY_OPT_MULTIPOLE:
+      if (value != 1 && value != 2) return fail(c, NBODY_EINVAL, "multipole order must be 1 or 2");
+      if (value == 2 && !c->tree.S64) {  // allocated on first use: 80 B per internal id
+        const size_t inner = size_t(1) << c->tree.L;
+        cudaError_t e = cudaMalloc(&c->quad_arena, 48 * inner + 32 * inner);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          c->quad_arena = nullptr;
+          return fail(c, NBODY_ENOMEM, "quadrupole arrays");
+        }
+        c->tree.S64 = reinterpret_cast<Quad64*>(c->quad_arena);
+        c->tree.qf = reinterpret_cast<float4*>(static_cast<char*>(c->quad_arena) + 48 * inner);
+      }
+      c->tree.quad = value == 2;
       drop_graph(c);
       return NBODY_OK;
     case NBODY_OPT_SORT_EVERY:
@@ -816,6 +833,16 @@ nbody_status nbody_debug_perm(nbody_ctx* c, uint32_t* perm) {
   return sync_stream(c);
 }
 
+nbody_status nbody_debug_quad(nbody_ctx* c, int level, double* S) {
+  CHECK_CTX(c);
+  if (level < 1 || level > c->tree.L) return fail(c, NBODY_EINVAL, "level out of range [1, L]");
+  if (!S) return fail(c, NBODY_EINVAL, "null output");
+  if (!c->tree.quad || !c->have_force) return fail(c, NBODY_ESTATE, "quadrupoles not enabled or not built");
+  CK(cudaMemcpyAsync(S, c->tree.S64 + c->tree.off[level], 48 * size_t(c->tree.count[level]), cudaMemcpyDefault,
+                     c->stream));
+  return sync_stream(c);
+}
+
 nbody_status nbody_debug_level(nbody_ctx* c, int level, int64_t* count, double* pred, float* rec, float* box) {
   CHECK_CTX(c);
   if (level < 1 || level > c->tree.L) return fail(c, NBODY_EINVAL, "level out of range [1, L]");
@@ -847,6 +874,7 @@ void nbody_destroy(nbody_ctx* c) {
   if (c->comm) ncclCommDestroy(c->comm);
 #endif
   if (c->arena) cudaFree(c->arena);
+  if (c->quad_arena) cudaFree(c->quad_arena);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
   if (c->cap_stream) cudaStreamDestroy(c->cap_stream);

@@ -23,10 +23,13 @@ struct GridInfo {
                  // R = max |coordinate| (K6)
 };
 
-// Balanced, ragged BVH stored level by level ([A6]).  Level 0 is the
-// sorted body array itself; internal node (l, j), l >= 1, lives at
-// off[l] + j of each per-node array (off[l] even, so sibling pairs are
-// 2-node aligned).
+// NEXT-4 [A24]: second mass moment about the COM, S = sum m (x-c)(x-c)^T.
+struct Quad64 {
+  double s[6];  // xx, yy, zz, xy, xz, yz (fp64, build + debug)
+};
+
+// Balanced, ragged BVH in heap numbering ([A6]): node (l, j) has id
+// off[l] + j with off[l] = 2^(L-l); leaf i is 2^L + i.
 struct TreeView {
   int L;                       // levels above the leaves
   int64_t n;                   // bodies (= nodes at level 0)
@@ -43,6 +46,9 @@ struct TreeView {
   double4* mom;    // (M, Mx, My, Mz) fp64 moments (build only) [A12]
   float4* blo;     // AABB lo (x, y, z, -)
   float4* bhi;     // AABB hi (x, y, z, -)
+  bool quad;       // NEXT-4: build second moments, add quadrupole terms
+  Quad64* S64;     // per internal node (quad only)
+  float4* qf;      // per internal node, 2 x float4: (Sxx, Syy, Szz, trS), (Sxy, Sxz, Syz, 0)
 };
 
 struct ForceParams {

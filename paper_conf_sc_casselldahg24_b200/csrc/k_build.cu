@@ -2,12 +2,18 @@
 // [A11] the whole body state moves) and K5 BUILDTREEACCUMULATEMASS (P:218,
 // P:221, Fig. 4; multipoles P:105).
 //
-// K5 is a parallel-for over the nodes of the next coarser level, level by
-// level, reducing the two children (left then right) -- the paper's
-// algorithm.  Moments (M, M x) are fp64 sums in that fixed order and the
-// boxes exact fp32 min/max, so every node record is bit-identical to the
-// oracle's [A12][A13][A16].  Per node it emits the opening-test record
-// (com64, s^2) and the fp32 monopole ((float)com64, (float)M) used by K6.
+// K5 reduces the two children of every node (left then right) level by
+// level -- the paper's algorithm.  Moments (M, M x) are fp64 sums in that
+// fixed order and the boxes exact fp32 min/max, so every node record is
+// bit-identical to the oracle's [A12][A13][A16].  Per node it emits the
+// opening-test record (com64, s^2), the fp32 filter thresholds and the fp32
+// monopole ((float)com64, (float)M) used by K6; with NEXT-4 also the second
+// moment about the COM (parallel-axis theorem, fp64, the oracle's operation
+// order) [A24].
+//
+// Default variant: a block reduces a 1024-leaf subtree (levels 1..10) in
+// shared memory and one block builds the top levels; variant 1 launches one
+// kernel per level (monopole only).  Both give identical records.
 #include "internal.cuh"
 
 namespace nb {
@@ -23,24 +29,32 @@ __global__ __launch_bounds__(256) void k_permute(const float4* __restrict__ pm_i
   vi_out[i] = __ldg(vi_in + p);
 }
 
-// Emit node `node`: the traversal records (pred, rec, rc) always; the build
-// moments and box only when `keep` (needed by a parent built in another
-// block, or by the debug views).
+// [A24] S_p += S_c + (M_c d_i) d_j, d = com_c - com_p, in the oracle's order.
+__device__ __forceinline__ void add_second_moment(double* Sp, const double* Sc, double Mc, const double* cc,
+                                                  const double* cp) {
+  const double d0 = __dsub_rn(cc[0], cp[0]), d1 = __dsub_rn(cc[1], cp[1]), d2 = __dsub_rn(cc[2], cp[2]);
+  const double di[6] = {d0, d1, d2, d0, d0, d1}, dj[6] = {d0, d1, d2, d1, d2, d2};
+#pragma unroll
+  for (int q = 0; q < 6; ++q) Sp[q] = __dadd_rn(Sp[q], __dadd_rn(Sc[q], __dmul_rn(__dmul_rn(Mc, di[q]), dj[q])));
+}
+
+// Emit node `node` with centre of mass c: the traversal records (pred, rec,
+// rc[, qf]) always; the build moments, box [and S64] only when `keep`
+// (needed by a parent built in another block, or by the debug views).
 __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, double M, double mx, double my, double mz,
-                                            float4 lo, float4 hi, bool keep = true) {
+                                            const double* c, float4 lo, float4 hi, bool keep,
+                                            const double* S = nullptr) {
   if (keep) {
     t.mom[node] = make_double4(M, mx, my, mz);
     t.blo[node] = lo;
     t.bhi[node] = hi;
   }
-  // centre of mass = first moment / mass [A12]
-  const double cx = __ddiv_rn(mx, M), cy = __ddiv_rn(my, M), cz = __ddiv_rn(mz, M);
   // [A3] s = longest side of the AABB (fp64 differences of fp32 bounds are exact)
   double s = __dsub_rn(double(hi.x), double(lo.x));
   s = fmax(s, __dsub_rn(double(hi.y), double(lo.y)));
   s = fmax(s, __dsub_rn(double(hi.z), double(lo.z)));
   const double s2 = __dmul_rn(s, s);
-  t.pred[node] = make_double4(cx, cy, cz, s2);
+  t.pred[node] = make_double4(c[0], c[1], c[2], s2);
   // Filter thresholds on the fp32 squared distance (DESIGN.md "fp32
   // filter"): |d2_fp32 - d^2| <= 1.01e-4 d^2 + A with A = 1e-9 R^2, so
   // d2 > (1 + 2e-4) s^2/theta^2 + A surely accepts and
@@ -55,7 +69,24 @@ __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, dou
     rc.x = rc.y = __int_as_float(0x7f800000);
   }
   t.rc[node] = rc;
-  t.rec[node] = make_float4(__double2float_rn(cx), __double2float_rn(cy), __double2float_rn(cz), __double2float_rn(M));
+  t.rec[node] =
+      make_float4(__double2float_rn(c[0]), __double2float_rn(c[1]), __double2float_rn(c[2]), __double2float_rn(M));
+  if (S) {
+    if (keep) {
+#pragma unroll
+      for (int q = 0; q < 6; ++q) t.S64[node].s[q] = S[q];
+    }
+    const float sxx = __double2float_rn(S[0]), syy = __double2float_rn(S[1]), szz = __double2float_rn(S[2]);
+    t.qf[2 * node] = make_float4(sxx, syy, szz, __double2float_rn(S[0] + S[1] + S[2]));
+    t.qf[2 * node + 1] = make_float4(__double2float_rn(S[3]), __double2float_rn(S[4]), __double2float_rn(S[5]), 0.f);
+  }
+}
+
+// centre of mass = first moment / mass [A12]
+__device__ __forceinline__ void node_com(double M, double mx, double my, double mz, double* c) {
+  c[0] = __ddiv_rn(mx, M);
+  c[1] = __ddiv_rn(my, M);
+  c[2] = __ddiv_rn(mz, M);
 }
 
 // Level 1 straight from the sorted bodies: leaf moments are M = m and
@@ -79,7 +110,9 @@ __global__ __launch_bounds__(256) void k_build_level1(TreeView t, const float4* 
     lo.x = fminf(lo.x, B.x); lo.y = fminf(lo.y, B.y); lo.z = fminf(lo.z, B.z);
     hi.x = fmaxf(hi.x, B.x); hi.y = fmaxf(hi.y, B.y); hi.z = fmaxf(hi.z, B.z);
   }
-  finish_node(t, t.off[1] + j, M, mx, my, mz, lo, hi);
+  double c[3];
+  node_com(M, mx, my, mz, c);
+  finish_node(t, t.off[1] + j, M, mx, my, mz, c, lo, hi, true);
 }
 
 // Level l >= 2 from level l - 1.
@@ -100,7 +133,9 @@ __global__ __launch_bounds__(256) void k_build_level(TreeView t, int l) {
     lo.x = fminf(lo.x, lb.x); lo.y = fminf(lo.y, lb.y); lo.z = fminf(lo.z, lb.z);
     hi.x = fmaxf(hi.x, hb.x); hi.y = fmaxf(hi.y, hb.y); hi.z = fmaxf(hi.z, hb.z);
   }
-  finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, lo, hi);
+  double c[3];
+  node_com(m.x, m.y, m.z, m.w, c);
+  finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, c, lo, hi, true);
 }
 
 // Fused build of levels 1..top (top <= 10) over a 1024-leaf subtree per
@@ -112,24 +147,34 @@ constexpr int kFuseLevels = 10;
 constexpr int kFuseHalf = 1 << (kFuseLevels - 1);  // level-1 nodes per block
 constexpr int kFuseThreads = 256;
 
+template <bool kQuad>
+constexpr int fuse_half() {  // level-1 nodes per block (quad: 512-leaf subtrees, 9 levels)
+  return kQuad ? kFuseHalf / 2 : kFuseHalf;
+}
+
+template <bool kQuad>
 __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const float4* __restrict__ leaves, int top,
                                                               bool keep_all) {
-  __shared__ double4 s_m[kFuseHalf];
-  __shared__ float4 s_lo[kFuseHalf];
-  __shared__ float4 s_hi[kFuseHalf];
+  constexpr int kHalf = kQuad ? kFuseHalf / 2 : kFuseHalf;
+  __shared__ double4 s_m[kHalf];
+  __shared__ float4 s_lo[kHalf];
+  __shared__ float4 s_hi[kHalf];
+  __shared__ double s_c[kQuad ? 3 * kHalf : 1];
+  __shared__ double s_S[kQuad ? 6 * kHalf : 1];
   const int64_t b = blockIdx.x;
-  for (int q = threadIdx.x; q < kFuseHalf; q += kFuseThreads) {
-    const int64_t j = b * kFuseHalf + q;
+  for (int q = threadIdx.x; q < kHalf; q += kFuseThreads) {
+    const int64_t j = b * kHalf + q;
     if (j >= t.count[1]) continue;
     const int64_t a = 2 * j;
     const float4 A = __ldg(leaves + a);
+    const bool two = a + 1 < t.n;
+    const float4 B = two ? __ldg(leaves + a + 1) : A;
     double M = double(A.w);
     double mx = __dmul_rn(double(A.w), double(A.x));
     double my = __dmul_rn(double(A.w), double(A.y));
     double mz = __dmul_rn(double(A.w), double(A.z));
     float4 lo = make_float4(A.x, A.y, A.z, 0.f), hi = lo;
-    if (a + 1 < t.n) {
-      const float4 B = __ldg(leaves + a + 1);
+    if (two) {
       M = __dadd_rn(M, double(B.w));
       mx = __dadd_rn(mx, __dmul_rn(double(B.w), double(B.x)));
       my = __dadd_rn(my, __dmul_rn(double(B.w), double(B.y)));
@@ -137,25 +182,45 @@ __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const 
       lo.x = fminf(lo.x, B.x); lo.y = fminf(lo.y, B.y); lo.z = fminf(lo.z, B.z);
       hi.x = fmaxf(hi.x, B.x); hi.y = fmaxf(hi.y, B.y); hi.z = fmaxf(hi.z, B.z);
     }
-    finish_node(t, t.off[1] + j, M, mx, my, mz, lo, hi, keep_all || top == 1);
+    double c[3];
+    node_com(M, mx, my, mz, c);
+    const bool keep = keep_all || top == 1;
+    if (kQuad) {
+      // leaves: com = position, S = 0 [A24]
+      const double zero[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+      double S[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+      const double ca[3] = {double(A.x), double(A.y), double(A.z)};
+      add_second_moment(S, zero, double(A.w), ca, c);
+      if (two) {
+        const double cb[3] = {double(B.x), double(B.y), double(B.z)};
+        add_second_moment(S, zero, double(B.w), cb, c);
+      }
+      finish_node(t, t.off[1] + j, M, mx, my, mz, c, lo, hi, keep, S);
+      for (int k = 0; k < 3; ++k) s_c[3 * q + k] = c[k];
+      for (int k = 0; k < 6; ++k) s_S[6 * q + k] = S[k];
+    } else {
+      finish_node(t, t.off[1] + j, M, mx, my, mz, c, lo, hi, keep);
+    }
     s_m[q] = make_double4(M, mx, my, mz);
     s_lo[q] = lo;
     s_hi[q] = hi;
   }
   __syncthreads();
   for (int l = 2; l <= top; ++l) {
-    const int cnt = kFuseHalf >> (l - 1);  // nodes of level l in this block (<= 256)
+    const int cnt = kHalf >> (l - 1);  // nodes of level l in this block (<= 256)
     const int q = threadIdx.x;
     const int64_t j = b * cnt + q;
     bool have = false;
     double4 m;
     float4 lo, hi;
+    double c[3], S[6];
     if (q < cnt && j < t.count[l]) {
       have = true;
+      const bool two = 2 * j + 1 < t.count[l - 1];
       m = s_m[2 * q];
       lo = s_lo[2 * q];
       hi = s_hi[2 * q];
-      if (2 * j + 1 < t.count[l - 1]) {
+      if (two) {
         const double4 mb = s_m[2 * q + 1];
         const float4 lb = s_lo[2 * q + 1], hb = s_hi[2 * q + 1];
         m.x = __dadd_rn(m.x, mb.x);
@@ -165,13 +230,26 @@ __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const 
         lo.x = fminf(lo.x, lb.x); lo.y = fminf(lo.y, lb.y); lo.z = fminf(lo.z, lb.z);
         hi.x = fmaxf(hi.x, hb.x); hi.y = fmaxf(hi.y, hb.y); hi.z = fmaxf(hi.z, hb.z);
       }
+      node_com(m.x, m.y, m.z, m.w, c);
+      if (kQuad) {
+        for (int k = 0; k < 6; ++k) S[k] = 0.0;
+        add_second_moment(S, &s_S[6 * (2 * q)], s_m[2 * q].x, &s_c[3 * (2 * q)], c);
+        if (two) add_second_moment(S, &s_S[6 * (2 * q + 1)], s_m[2 * q + 1].x, &s_c[3 * (2 * q + 1)], c);
+      }
     }
     __syncthreads();
     if (have) {
       s_m[q] = m;
       s_lo[q] = lo;
       s_hi[q] = hi;
-      finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, lo, hi, keep_all || l == top);
+      const bool keep = keep_all || l == top;
+      if (kQuad) {
+        for (int k = 0; k < 3; ++k) s_c[3 * q + k] = c[k];
+        for (int k = 0; k < 6; ++k) s_S[6 * q + k] = S[k];
+        finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, c, lo, hi, keep, S);
+      } else {
+        finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, c, lo, hi, keep);
+      }
     }
     __syncthreads();
   }
@@ -183,9 +261,10 @@ __global__ __launch_bounds__(1024) void k_build_upper(TreeView t, int from) {
   for (int l = from; l <= t.L; ++l) {
     for (int64_t j = threadIdx.x; j < t.count[l]; j += blockDim.x) {
       const int64_t ca = t.off[l - 1] + 2 * j;
+      const bool two = 2 * j + 1 < t.count[l - 1];
       double4 m = t.mom[ca];
       float4 lo = t.blo[ca], hi = t.bhi[ca];
-      if (2 * j + 1 < t.count[l - 1]) {
+      if (two) {
         const double4 mb = t.mom[ca + 1];
         const float4 lb = t.blo[ca + 1], hb = t.bhi[ca + 1];
         m.x = __dadd_rn(m.x, mb.x);
@@ -195,7 +274,22 @@ __global__ __launch_bounds__(1024) void k_build_upper(TreeView t, int from) {
         lo.x = fminf(lo.x, lb.x); lo.y = fminf(lo.y, lb.y); lo.z = fminf(lo.z, lb.z);
         hi.x = fmaxf(hi.x, hb.x); hi.y = fmaxf(hi.y, hb.y); hi.z = fmaxf(hi.z, hb.z);
       }
-      finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, lo, hi, true);
+      double c[3];
+      node_com(m.x, m.y, m.z, m.w, c);
+      if (t.quad) {
+        double S[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+        const double4 pa = t.pred[ca];
+        const double cca[3] = {pa.x, pa.y, pa.z};
+        add_second_moment(S, t.S64[ca].s, t.mom[ca].x, cca, c);
+        if (two) {
+          const double4 pb = t.pred[ca + 1];
+          const double ccb[3] = {pb.x, pb.y, pb.z};
+          add_second_moment(S, t.S64[ca + 1].s, t.mom[ca + 1].x, ccb, c);
+        }
+        finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, c, lo, hi, true, S);
+      } else {
+        finish_node(t, t.off[l] + j, m.x, m.y, m.z, m.w, c, lo, hi, true);
+      }
     }
     __syncthreads();
   }
@@ -205,9 +299,14 @@ __global__ __launch_bounds__(1024) void k_build_upper(TreeView t, int from) {
 
 void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, cudaStream_t s) {
   if (t.L < 1) return;
-  const int top = t.L < kFuseLevels ? t.L : kFuseLevels;
-  const unsigned grid = unsigned((t.count[1] + kFuseHalf - 1) / kFuseHalf);
-  k_build_fused<<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
+  const int levels = t.quad ? kFuseLevels - 1 : kFuseLevels;
+  const int half = t.quad ? fuse_half<true>() : fuse_half<false>();
+  const int top = t.L < levels ? t.L : levels;
+  const unsigned grid = unsigned((t.count[1] + half - 1) / half);
+  if (t.quad)
+    k_build_fused<true><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
+  else
+    k_build_fused<false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
   if (t.L > top) k_build_upper<<<1, 1024, 0, s>>>(t, top + 1);
 }
 

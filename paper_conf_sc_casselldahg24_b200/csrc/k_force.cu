@@ -97,6 +97,27 @@ struct Acc {
   }
 };
 
+// NEXT-4 [A24]: the quadrupole term of internal node qid (the oracle's
+// interact_quad in fp32): with d = com - x, inv = (|d|^2 + eps^2)^(-1/2),
+//   a += [(15/2) d.S.d inv^7 - (3/2) tr(S) inv^5] d - 3 (S d) inv^5.
+// qf[2 qid] = (Sxx, Syy, Szz, trS), qf[2 qid + 1] = (Sxy, Sxz, Syz, 0).
+__device__ __forceinline__ void quad_term(Acc& a, float dx, float dy, float dz, float inv,
+                                          const float4* __restrict__ qf, uint32_t qid, bool on) {
+  const float4 q0 = __ldg(qf + 2 * size_t(qid)), q1 = __ldg(qf + 2 * size_t(qid) + 1);
+  const float inv2 = inv * inv;
+  const float inv5 = inv2 * inv2 * inv;
+  const float inv7 = inv5 * inv2;
+  const float sx = fmaf(q0.x, dx, fmaf(q1.x, dy, q1.y * dz));
+  const float sy = fmaf(q1.x, dx, fmaf(q0.y, dy, q1.z * dz));
+  const float sz = fmaf(q1.y, dx, fmaf(q1.z, dy, q0.z * dz));
+  const float dsd = fmaf(dx, sx, fmaf(dy, sy, dz * sz));
+  const float c = on ? fmaf(7.5f * dsd, inv7, -1.5f * q0.w * inv5) : 0.f;
+  const float e = on ? -3.f * inv5 : 0.f;
+  a.x = fmaf(c, dx, fmaf(e, sx, a.x));
+  a.y = fmaf(c, dy, fmaf(e, sy, a.y));
+  a.z = fmaf(c, dz, fmaf(e, sz, a.z));
+}
+
 struct Probe {
   float dx, dy, dz, d2;
 };
@@ -116,6 +137,7 @@ struct Walk {
   const float4* rc2;     // rc viewed as pairs (lo_A, hi_A, lo_B, hi_B)
   const float2* rc;
   const double4* pred;
+  const float4* qf;      // NEXT-4 quadrupoles (2 float4 per id) or null
   uint32_t leaf0, n;
   int L;
 };
@@ -132,6 +154,7 @@ __device__ __forceinline__ Walk make_walk(const ForceParams& P) {
   W.rc = in_reg(P.t.rc);
   W.rc2 = reinterpret_cast<const float4*>(W.rc);
   W.pred = in_reg(P.t.pred);
+  W.qf = P.t.qf;
   W.L = P.t.L;
   W.leaf0 = 1u << W.L;
   W.n = uint32_t(P.t.n);
@@ -150,6 +173,14 @@ __device__ __forceinline__ bool decide1(const Walk& W, uint32_t g, bool in, floa
 
 // The per-lane mask-stack walk of the subtree of node g0 for the lanes in
 // mask0 (all of which reached g0).
+// NEXT-4: quadrupole of an accepted internal node in the mask walk.
+__device__ __forceinline__ void quad_at(Acc& a, const Probe& p, float eps2, const float4* qf, uint32_t g, bool on) {
+  const float r2 = p.d2 + eps2;
+  const float inv = r2 > 0.f ? rsqrt_fast(r2) : 0.f;
+  quad_term(a, p.dx, p.dy, p.dz, inv, qf, g, on);
+}
+
+template <bool kQuad>
 __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32_t kid, Acc& a, int lane, uint32_t g0,
                                           uint32_t mask0) {
   // the start node on its own
@@ -164,7 +195,10 @@ __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32
       return;
     }
     const bool acc = decide1(W, g0, in, p.d2, __ldg(W.rc + g0), T);
-    if (__any_sync(kFull, acc)) a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+    if (__any_sync(kFull, acc)) {
+      a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+      if (kQuad) quad_at(a, p, T.eps2, W.qf, g0, acc);
+    }
     a.n += acc;
     const uint32_t rej = __ballot_sync(kFull, in && !acc);
     if (rej == 0) return;
@@ -208,8 +242,14 @@ __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32
       if (pushA && lane == q) { sg = 2u * g; sm = rejA; }
       sp = q + int(pushA);
     }
-    if (__any_sync(kFull, accA)) a.add(accA, pA.dx, pA.dy, pA.dz, pA.d2, rA.w, T.eps2);
-    if (__any_sync(kFull, accB)) a.add(accB, pB.dx, pB.dy, pB.dz, pB.d2, rB.w, T.eps2);
+    if (__any_sync(kFull, accA)) {
+      a.add(accA, pA.dx, pA.dy, pA.dz, pA.d2, rA.w, T.eps2);
+      if (kQuad && l > 0) quad_at(a, pA, T.eps2, W.qf, g, accA);
+    }
+    if (__any_sync(kFull, accB)) {
+      a.add(accB, pB.dx, pB.dy, pB.dz, pB.d2, rB.w, T.eps2);
+      if (kQuad && l > 0) quad_at(a, pB, T.eps2, W.qf, g + 1u, accB);
+    }
     a.n += accA;
     a.n += accB;
   }
@@ -238,6 +278,7 @@ __device__ __forceinline__ void store_result(const ForceParams& P, int64_t k, bo
 // ------------------------------------------------------------ variant 1 ----
 constexpr int kV1Warps = 8;
 
+template <bool kQuad>
 __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForceParams P) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t k = P.t_begin + (int64_t(blockIdx.x) * kV1Warps + w) * 32 + lane;
@@ -248,7 +289,7 @@ __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForcePa
   Acc a;
   const Walk W = make_walk(P);
   const uint32_t kid = W.leaf0 + uint32_t(k);
-  mask_walk(W, T, kid, a, lane, 1u, amask);
+  mask_walk<kQuad>(W, T, kid, a, lane, 1u, amask);
   store_result(P, k, active, a, lane);
 }
 
@@ -275,6 +316,7 @@ constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 constexpr int kCapF = NBODY_CAP_F;  // dense list: entries every active lane interacts with
 constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 
+template <bool kQuad>
 struct V0Smem {
   float4 tgt[32];        // the warp's target positions
   float4 frec[kCapF];    // monopole / body records, all lanes
@@ -282,6 +324,8 @@ struct V0Smem {
   uint32_t pmsk[kCapP];  // ... for the lanes in the mask
   uint32_t astk[kCapA];
   uint2 tstk[kCapT];     // (id, mask of the targets that reached it)
+  uint32_t fid[kQuad ? kCapF : 1];  // NEXT-4: node id of each entry (0: a body)
+  uint32_t pid[kQuad ? kCapP : 1];
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -296,8 +340,10 @@ __device__ __forceinline__ float warp_maxf(float v) {
 }
 
 // a += m r / (|r|^2 + eps^2)^(3/2), r = s - x.  kSoft (eps > 0): r2 > 0 always.
-template <bool kSoft>
-__device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const Target& T) {
+// kQuad with qid != 0 (warp-uniform): plus node qid's quadrupole [A24].
+template <bool kSoft, bool kQuad>
+__device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const Target& T, const float4* qf,
+                                         uint32_t qid, bool on) {
   const float dx = s.x - T.x, dy = s.y - T.y, dz = s.z - T.z;
   const float r2 = fmaf(dz, dz, fmaf(dy, dy, fmaf(dx, dx, T.eps2)));
   float inv = rsqrt_fast(r2);
@@ -306,34 +352,38 @@ __device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const
   a.x = fmaf(w, dx, a.x);
   a.y = fmaf(w, dy, a.y);
   a.z = fmaf(w, dz, a.z);
+  if (kQuad && qid) quad_term(a, dx, dy, dz, inv, qf, qid, on);
 }
 
-template <bool kSoft>
-__device__ __forceinline__ void dense_full(const V0Smem& S, int nf, const Target& T, Acc& a) {
+template <bool kSoft, bool kQuad>
+__device__ __forceinline__ void dense_full(const V0Smem<kQuad>& S, int nf, const Target& T, Acc& a,
+                                           const float4* qf) {
 #pragma unroll 4
   for (int e = 0; e < nf; ++e) {
     const float4 s = S.frec[e];
-    interact<kSoft>(a, s, s.w, T);
+    interact<kSoft, kQuad>(a, s, s.w, T, qf, kQuad ? S.fid[e] : 0u, true);
   }
   a.n += uint32_t(nf);
 }
 
-template <bool kSoft>
-__device__ __forceinline__ void dense_part(const V0Smem& S, int np, const Target& T, Acc& a, int lane) {
+template <bool kSoft, bool kQuad>
+__device__ __forceinline__ void dense_part(const V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane,
+                                           const float4* qf) {
 #pragma unroll 4
   for (int e = 0; e < np; ++e) {
     const float4 s = S.prec[e];
     const bool on = (S.pmsk[e] >> lane) & 1u;
-    interact<kSoft>(a, s, on ? s.w : 0.f, T);
+    interact<kSoft, kQuad>(a, s, on ? s.w : 0.f, T, qf, kQuad ? S.pid[e] : 0u, on);
     a.n += on;
   }
 }
 
-template <bool kSoft>
+template <bool kSoft, bool kQuad>
 __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(const ForceParams P) {
-  __shared__ V0Smem s_all[kV0Warps];
+  __shared__ V0Smem<kQuad> s_all[kV0Warps];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  V0Smem& S = s_all[w];
+  V0Smem<kQuad>& S = s_all[w];
+  const float4* qf = kQuad ? in_reg(P.t.qf) : nullptr;
   const int64_t k0 = P.t_begin + (int64_t(blockIdx.x) * kV0Warps + w) * 32;
   const int64_t k = k0 + lane;
   const bool active = k < P.t_end;
@@ -362,16 +412,22 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
 
   // Append (record r, lane mask msk) to the dense lists: full when every
   // active lane interacts with it.
-  auto append = [&](bool want, const float4& r, uint32_t msk) {
+  // active lane interacts with it.  id: the node (quadrupole source), 0 for a body.
+  auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id) {
     const bool full = want && msk == amask;
     const bool part = want && msk != amask;
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
-    if (full) S.frec[nf + __popc(bf & lt)] = r;
+    if (full) {
+      const int pos = nf + __popc(bf & lt);
+      S.frec[pos] = r;
+      if (kQuad) S.fid[pos] = id;
+    }
     if (part) {
       const int pos = np + __popc(bp & lt);
       S.prec[pos] = r;
       S.pmsk[pos] = msk;
+      if (kQuad) S.pid[pos] = id;
     }
     nf += __popc(bf);
     np += __popc(bp);
@@ -379,11 +435,11 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   auto flush = [&](bool all) {
     __syncwarp();
     if (nf > kCapF - 32 || (all && nf > 0)) {
-      dense_full<kSoft>(S, nf, T, a);
+      dense_full<kSoft, kQuad>(S, nf, T, a, qf);
       nf = 0;
     }
     if (np > kCapP - 32 || (all && np > 0)) {
-      dense_part<kSoft>(S, np, T, a, lane);
+      dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
       np = 0;
     }
     __syncwarp();
@@ -425,7 +481,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
         }
       }
       if (g >= leaf0 && g - kid0 < 32u) am &= ~(1u << (g - kid0));  // a leaf never acts on itself
-      append(am != 0u, r, am);
+      append(am != 0u, r, am, g < leaf0 ? g : 0u);
       // children of opened nodes, with the mask of the targets that opened them
       const int l = L - 31 + __clz(int(g));
       const bool two = rm && (((2u * g + 1u) << (l - 1)) - leaf0) < n;
@@ -447,9 +503,9 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
         spill &= spill - 1u;
         const uint32_t gs = __shfl_sync(kFull, g, src);
         const uint32_t ms = __shfl_sync(kFull, rm, src);
-        mask_walk(W, T, kid, a, lane, 2u * gs, ms);
+        mask_walk<kQuad>(W, T, kid, a, lane, 2u * gs, ms);
         const int ls = L - 31 + __clz(int(gs));
-        if ((((2u * gs + 1u) << (ls - 1)) - leaf0) < n) mask_walk(W, T, kid, a, lane, 2u * gs + 1u, ms);
+        if ((((2u * gs + 1u) << (ls - 1)) - leaf0) < n) mask_walk<kQuad>(W, T, kid, a, lane, 2u * gs + 1u, ms);
       }
     } else if (na > 0) {
       // ---- A: box classification of up to 32 nodes reached by every lane
@@ -498,7 +554,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       }
       uint32_t msk = amask;
       if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
-      append(cls == 1, r, msk);
+      append(cls == 1, r, msk, g < leaf0 ? g : 0u);
       const uint32_t bt = __ballot_sync(kFull, cls == 3);
       if (cls == 3) S.tstk[nt + __popc(bt & lt)] = make_uint2(g, amask);
       nt += __popc(bt);
@@ -525,15 +581,24 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
   const int64_t nt = p.t_end - p.t_begin;
   if (nt <= 0) return;
   const int64_t warps = (nt + 31) / 32;
+  const bool quad = p.t.quad;
   if (variant == 1) {
     const unsigned grid = unsigned((warps + kV1Warps - 1) / kV1Warps);
-    k_force_maskstack<<<grid, 32 * kV1Warps, 0, s>>>(p);
+    if (quad)
+      k_force_maskstack<true><<<grid, 32 * kV1Warps, 0, s>>>(p);
+    else
+      k_force_maskstack<false><<<grid, 32 * kV1Warps, 0, s>>>(p);
   } else {
     const unsigned grid = unsigned((warps + kV0Warps - 1) / kV0Warps);
-    if (p.eps2 > 0.f)
-      k_force_grouped<true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    const bool soft = p.eps2 > 0.f;
+    if (soft && !quad)
+      k_force_grouped<true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    else if (!soft && !quad)
+      k_force_grouped<false, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    else if (soft)
+      k_force_grouped<true, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
     else
-      k_force_grouped<false><<<grid, 32 * kV0Warps, 0, s>>>(p);
+      k_force_grouped<false, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
   }
 }
 

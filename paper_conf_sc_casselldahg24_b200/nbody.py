@@ -46,7 +46,7 @@ class NBody:
     """One simulation context: ``NBody(n, theta, eps, dt)``."""
 
     def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
-                 stream=None, use_graph: bool = True, traversal: int = 0, device=None):
+                 stream=None, use_graph: bool = True, traversal: int = 0, device=None, multipole: int = 1):
         self.lib = _capi.load()
         self.n = int(n)
         if device is None:  # follow PyTorch's current device when torch has one
@@ -68,6 +68,8 @@ class NBody:
         self.set_option(_capi.NBODY_OPT_KEY_BITS, key_bits)
         self.set_option(_capi.NBODY_OPT_USE_GRAPH, int(use_graph))
         self.set_option(_capi.NBODY_OPT_TRAVERSAL, traversal)
+        if multipole != 1:
+            self.set_option(_capi.NBODY_OPT_MULTIPOLE, multipole)
         if stream is not None:
             self.set_option(_capi.NBODY_OPT_STREAM, int(stream))
 
@@ -178,6 +180,13 @@ class NBody:
     def debug_perm(self):
         out = np.empty(self.n, np.uint32)
         self._ck(self.lib.nbody_debug_perm(self.h, _ptr(out)))
+        return out
+
+    def debug_quad(self, level: int):
+        cnt = C.c_int64()
+        self._ck(self.lib.nbody_debug_level(self.h, int(level), C.byref(cnt), None, None, None))
+        out = np.empty((cnt.value, 6), np.float64)
+        self._ck(self.lib.nbody_debug_quad(self.h, int(level), _ptr(out)))
         return out
 
     def debug_level(self, level: int):

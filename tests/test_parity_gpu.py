@@ -323,3 +323,37 @@ def test_tree_reuse_against_oracle(NB, oracle):
     assert_acc_close(acc, r1.acc)
     cnt = s.get_interactions()[r1.ids]
     assert np.mean(cnt == r1.count) > 0.99
+
+
+# --------------------------------------------------- NEXT-4 quadrupoles ------
+@pytest.mark.parametrize("name,n,seed,theta", [("plummer", 20_000, 93, 0.5), ("disks", 30_001, 94, 0.8),
+                                               ("clustered", 1025, 95, 0.6), ("uniform", 3, 96, 0.5)])
+def test_quadrupole_parity(NB, oracle, name, n, seed, theta):
+    pos, vel, mass = generate(name, n, seed)
+    sim = NB(n, theta, EPS, DT, multipole=2)
+    sim.set_bodies(pos, vel, mass)
+    sim.compute_accel()
+    ref = oracle.step(pos, vel, mass, theta=theta, eps=EPS, dt=DT, integrate=False, quad=True)
+    for l in range(1, ref.tree.L + 1):  # second moments bit-exact [A24]
+        assert (sim.debug_quad(l) == ref.tree.level_quad(l)).all(), l
+    assert (sim.get_interactions()[ref.ids] == ref.count).all()
+    assert_acc_close(sim.get_accel()[ref.ids], ref.acc)
+    v1 = NB(n, theta, EPS, DT, multipole=2, traversal=1)  # mask-walk variant
+    v1.set_bodies(pos, vel, mass)
+    v1.compute_accel()
+    assert (v1.get_interactions() == sim.get_interactions()).all()
+    assert rel_errors(v1.get_accel(), sim.get_accel()).max() < 1e-4
+
+
+def test_quadrupole_is_more_accurate_at_1M(NB):
+    n = 1_000_000
+    pos, vel, mass = generate("plummer", n, 2)
+    ids = np.random.default_rng(97).choice(n, 500, replace=False)
+    errs = {}
+    for mp in (1, 2):
+        sim = NB(n, 0.5, EPS, DT, multipole=mp)
+        sim.set_bodies(pos, vel, mass)
+        sim.compute_accel()
+        exact = sim.direct_accel(ids)
+        errs[mp] = float(np.sqrt(np.mean(rel_errors(sim.get_accel()[ids], exact) ** 2)))
+    assert errs[2] < 0.5 * errs[1], errs
