@@ -110,9 +110,14 @@ __global__ __launch_bounds__(kThreads, 2) void k_onesweep(const K* __restrict__ 
   }
   // Rank inside the warp, in (item, lane) order = position order: stable.
   uint32_t* wh = s_whist + w * kRadix;
+  // all matches first (independent, so their latencies overlap) ...
+  uint32_t pm[kItems];
+#pragma unroll
+  for (int i = 0; i < kItems; ++i) pm[i] = __match_any_sync(0xffffffffu, d[i]);
+  // ... then the per-warp digit counters, item by item
 #pragma unroll
   for (int i = 0; i < kItems; ++i) {
-    const uint32_t peers = __match_any_sync(0xffffffffu, d[i]);
+    const uint32_t peers = pm[i];
     const int leader = __ffs(peers) - 1;
     const uint32_t below = __popc(peers & ((1u << lane) - 1u));
     uint32_t pre = 0;
@@ -145,15 +150,34 @@ __global__ __launch_bounds__(kThreads, 2) void k_onesweep(const K* __restrict__ 
       s_dglobal[tid] = gb;
     } else {
       mine.store(kFlagAgg | cnt, cuda::memory_order_relaxed);
+      // Windowed look-back: the status words of up to 8 predecessors are
+      // loaded at once (one L2 round trip), then consumed in order; an
+      // unpublished one is re-polled; an inclusive prefix ends the walk.
+      constexpr int kWin = 8;
       uint32_t excl = 0;
       int64_t p = tile - 1;
-      for (;;) {
-        cuda::atomic_ref<uint32_t, cuda::thread_scope_device> o(status[p * kRadix + tid]);
-        const uint32_t s = o.load(cuda::memory_order_relaxed);
-        if ((s & ~kValMask) == 0) continue;  // predecessor not published yet
-        excl += s & kValMask;
-        if (s & kFlagInc) break;
-        --p;
+      bool done = false;
+      while (!done) {
+        const int wn = p + 1 < kWin ? int(p + 1) : kWin;
+        uint32_t sv[kWin];
+#pragma unroll
+        for (int i = 0; i < kWin; ++i)
+          if (i < wn) {
+            cuda::atomic_ref<uint32_t, cuda::thread_scope_device> o(status[(p - i) * kRadix + tid]);
+            sv[i] = o.load(cuda::memory_order_relaxed);
+          }
+#pragma unroll
+        for (int i = 0; i < kWin; ++i) {
+          if (done || i >= wn) continue;
+          uint32_t s = sv[i];
+          while ((s & ~kValMask) == 0) {  // predecessor not published yet
+            cuda::atomic_ref<uint32_t, cuda::thread_scope_device> o(status[(p - i) * kRadix + tid]);
+            s = o.load(cuda::memory_order_relaxed);
+          }
+          excl += s & kValMask;
+          if (s & kFlagInc) done = true;
+        }
+        p -= wn;
       }
       mine.store(kFlagInc | (excl + cnt), cuda::memory_order_relaxed);
       s_dglobal[tid] = gb + excl;
