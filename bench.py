@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle force-sample time")
+    ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
+                    help="multi-GPU exchange: fused update + peer-memory stores (default) or NCCL all-gather")
     ap.add_argument("--sort-every", type=int, default=1,
                     help="ablation: tree reuse, re-sort every k-th step (NEXT-3(iii)); 1 = Alg. 6")
     return ap.parse_args()
@@ -67,7 +69,7 @@ def workload(args):
 def config_json(cfg, world, extra=None):
     d = {"workload": f"{cfg['workload']} N={cfg['n']} ({args_config_name(cfg)})", "n": cfg["n"],
          "theta": cfg["theta"], "eps": cfg["eps"], "dt": cfg["dt"], "key_bits": 16, "seed": cfg["seed"],
-         "sort_every": cfg.get("sort_every", 1),
+         "sort_every": cfg.get("sort_every", 1), "exchange": cfg.get("exchange", "none"),
          "parallelism": "single" if world == 1 else f"hilbert-range x{world}",
          "l2": "inputs larger than L2 (bodies 320 MB + tree ~1 GB per step at N=1e7); no explicit flush"}
     if extra:
@@ -219,7 +221,11 @@ def run_ours(args, cfg, world, rank, local):
         sim.set_option(7, args.sort_every)  # NBODY_OPT_SORT_EVERY
         cfg["sort_every"] = args.sort_every
     if world > 1:
-        sim.attach_process_group(rank, world)
+        if args.exchange == "peer" and world <= 8:
+            sim.attach_peers_group(rank, world)
+        else:
+            sim.attach_process_group(rank, world)
+        cfg["exchange"] = sim.exchange_mode()
     sim.set_bodies(pos, vel, mass)
 
     def barrier():

@@ -199,6 +199,36 @@ nbody_status nbody_get_partition(nbody_ctx *ctx, int *rank, int *world, int64_t 
  * world): the exchange step of an emulated partition. */
 nbody_status nbody_copy_owned(nbody_ctx *dst, nbody_ctx *src);
 
+/* ---- fused update + exchange over peer memory ------------
+ * The alternative to the NCCL all-gather for up to 8 ranks in one NVLink /
+ * NVSwitch domain: every rank maps every other rank's state buffers, and the
+ * leapfrog kernel (K7 of Alg. 6) stores each updated record of
+ * its Hilbert range [A21] straight into the same slot of ALL ranks' state,
+ * so the exchange is the update's own stores.  Two device-side barriers per
+ * step (flags in each rank's memory, release/acquire at system scope) order
+ * the stores against the readers; a barrier that waits > 20 s (a rank that
+ * stopped stepping) marks the context failed (NBODY_ESTATE from the next
+ * synchronising call).  Results are bit-identical to one GPU.  All ranks
+ * must call nbody_step / nbody_compute_accel the same number of times;
+ * by-id getters are NOT collective in this mode (they read the peers'
+ * forces directly).  Contexts must be destroyed together. */
+
+/* Write this context's 128-byte peer descriptor (a CUDA IPC handle of its
+ * device arena plus N and the layout size) for the other ranks. */
+nbody_status nbody_peer_handle(nbody_ctx *ctx, void *out128);
+/* Map the peers: handles = world descriptors of 128 bytes, indexed by rank
+ * (gathered by the caller, e.g. all_gather over torch.distributed), world
+ * <= 8, every rank in its own process.  Partitions the context as
+ * (rank, world) and selects the fused exchange.  Not with NCCL attached. */
+nbody_status nbody_attach_peers(nbody_ctx *ctx, const void *handles128, int rank, int world);
+/* The same for `world` contexts of ONE process (ctxs[r] becomes rank r), on
+ * one device (single-GPU emulation of the exchange) or on several (peer
+ * access is enabled). */
+nbody_status nbody_attach_peers_local(nbody_ctx **ctxs, int world);
+/* 0 = no exchange (single rank or emulated partition), 1 = NCCL all-gather,
+ * 2 = fused peer-memory exchange; -1 for a null context. */
+int nbody_exchange_mode(nbody_ctx *ctx);
+
 /* ---- debug views of the last force pass (parity tests) ---------------- */
 /* Hilbert keys of the bodies in the slot order BEFORE the last sort:
  * keys[n] as uint64 (3b bits, Skilling's index). */

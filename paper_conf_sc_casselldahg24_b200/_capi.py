@@ -73,6 +73,10 @@ SIGNATURES = {
     "nbody_get_partition": (_S, [_P, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(_I64),
                                  C.POINTER(_I64)]),
     "nbody_copy_owned": (_S, [_P, _P]),
+    "nbody_peer_handle": (_S, [_P, _P]),
+    "nbody_attach_peers": (_S, [_P, _P, C.c_int, C.c_int]),
+    "nbody_attach_peers_local": (_S, [C.POINTER(_P), C.c_int]),
+    "nbody_exchange_mode": (C.c_int, [_P]),
     "nbody_debug_quad": (_S, [_P, C.c_int, _P]),
     "nbody_debug_keys": (_S, [_P, _P]),
     "nbody_debug_perm": (_S, [_P, _P]),

@@ -82,6 +82,16 @@ struct nbody_ctx {
 #ifdef NBODY_WITH_NCCL
   ncclComm_t comm = nullptr;
 #endif
+  // fused K7 + exchange over peer memory (k_exchange.cu)
+  size_t arena_bytes = 0;
+  bool xpeer = false;
+  PeerTable peers{};
+  const float4* peer_acc[kMaxPeers] = {};
+  const uint32_t* peer_cnt[kMaxPeers] = {};
+  void* peer_map[kMaxPeers] = {};   // CUDA IPC mappings to close
+  unsigned* xflags = nullptr;       // [kBarrierSlots][kMaxPeers] epochs signalled to this rank
+  unsigned* xepoch = nullptr;       // [kBarrierSlots] this rank's barrier counters
+  int* xerr = nullptr;              // set by a barrier that timed out
 };
 
 namespace {
@@ -202,6 +212,7 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 16 * size_t(inner);                     // blo
   sz[k++] = 16 * size_t(inner);                     // bhi
   sz[k++] = 8 * size_t(ids);                        // rc (-inf at the leaves)
+  sz[k++] = 256;                                    // exchange flags, epochs, error
   size_t total = 0;
   for (int i = 0; i < k; ++i) total += align_up(sz[i]);
   cudaError_t e = cudaMalloc(&c->arena, total);
@@ -237,6 +248,10 @@ nbody_status allocate(nbody_ctx* c) {
   c->tree.blo = (float4*)take();
   c->tree.bhi = (float4*)take();
   c->tree.rc = (float2*)take();
+  c->xflags = (unsigned*)take();
+  c->xepoch = c->xflags + kBarrierSlots * kMaxPeers;
+  c->xerr = reinterpret_cast<int*>(c->xepoch + kBarrierSlots);
+  c->arena_bytes = total;
   c->tree.grid = c->grid;
   c->tree.th2 = c->theta * c->theta;
   // the sorted bodies live in the leaf ids of the record array
@@ -244,7 +259,8 @@ nbody_status allocate(nbody_ctx* c) {
   // leaves always interact when reached: thresholds (-inf, -inf), set once
   const float ninf = -INFINITY;
   launch_fill_float2(c->tree.rc + (int64_t(1) << c->tree.L), n, make_float2(ninf, ninf), nullptr);
-  e = cudaDeviceSynchronize();
+  e = cudaMemset(c->xflags, 0, 256);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
   c->sort.n = n;
   c->sort.tiles = tiles;
@@ -301,6 +317,11 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     CK(cudaMemcpyAsync(c->vi[1], c->vi[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
   }
   c->last_sorted = resort;
+  int x_kernels = 0;
+  if (c->xpeer && integrate) {  // every rank has consumed the old state: peers may overwrite it
+    launch_xbarrier(c->peers, c->xepoch, 0, c->xerr, s);
+    ++x_kernels;
+  }
   int build_kernels;
   if (c->build_variant == 1 && !c->tree.quad) {  // the level-by-level variant is monopole only
     launch_build(c->tree, c->pm[1], s);
@@ -326,7 +347,13 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   fp.total = c->total;
   launch_force(fp, c->traversal, s);
   CK(mark(4));
-  if (integrate) {
+  if (integrate && c->xpeer) {
+    // K7 stores the owned records into every rank's state, then the
+    // delivery barrier (k_exchange.cu)
+    launch_leapfrog_scatter(c->pm[1], c->vi[1], c->acc, ob, oe - ob, float(c->dt), c->peers, s);
+    launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
+    ++x_kernels;
+  } else if (integrate) {
     launch_leapfrog(c->pm[1] + ob, c->vi[1] + ob, c->acc, oe - ob, float(c->dt), c->pm[0] + ob, c->vi[0] + ob, s);
 #ifdef NBODY_WITH_NCCL
     if (c->comm) {  // S0 of the next step: every rank gets every owned slice
@@ -344,11 +371,15 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   } else {
     CK(cudaMemcpyAsync(c->pm[0], c->pm[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
     CK(cudaMemcpyAsync(c->vi[0], c->vi[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    if (c->xpeer) {  // every rank's forces are final before a getter reads them
+      launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
+      ++x_kernels;
+    }
   }
   CK(mark(5));
   c->ev_valid = tm;
   // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 + K6 1 + K7 1
-  c->kernels_per_step = front_kernels + build_kernels + 1 + (integrate ? 1 : 0);
+  c->kernels_per_step = front_kernels + build_kernels + 1 + (integrate ? 1 : 0) + x_kernels;
   CK(cudaGetLastError());
   return NBODY_OK;
 }
@@ -373,8 +404,45 @@ nbody_status build_graph(nbody_ctx* c, bool resort) {
 
 nbody_status sync_stream(nbody_ctx* c) {
   CK(cudaStreamSynchronize(c->stream));
+  if (c->xpeer) {
+    int err = 0;
+    CK(cudaMemcpy(&err, c->xerr, sizeof(int), cudaMemcpyDeviceToHost));
+    if (err) {
+      c->state = NBODY_ESTATE;
+      c->err = "peer exchange: a barrier timed out (a rank stopped stepping); the state is invalid";
+      return NBODY_ESTATE;
+    }
+  }
   return NBODY_OK;
 }
+
+// Fill the peer table from every rank's arena base (layouts are identical:
+// same N, same plan) and switch the context to the fused exchange.
+void attach_peer_bases(nbody_ctx* c, char* const* base, int rank, int world) {
+  auto at = [&](int q, const void* own) { return base[q] + (static_cast<const char*>(own) - c->arena); };
+  PeerTable& pt = c->peers;
+  pt.G = world;
+  pt.rank = rank;
+  for (int q = 0; q < world; ++q) {
+    pt.pm[q] = (float4*)at(q, c->pm[0]);
+    pt.vi[q] = (float4*)at(q, c->vi[0]);
+    pt.flags[q] = (unsigned*)at(q, c->xflags);
+    c->peer_acc[q] = (const float4*)at(q, c->acc);
+    c->peer_cnt[q] = (const uint32_t*)at(q, c->cnt);
+  }
+  set_part(c, rank, world);
+  c->xpeer = true;
+  drop_graph(c);
+}
+
+struct PeerDesc {  // nbody_peer_handle's 128-byte record
+  cudaIpcMemHandle_t ipc;
+  int64_t n;
+  uint64_t arena_bytes;
+  uint32_t magic;
+};
+static_assert(sizeof(PeerDesc) <= 128, "peer descriptor must fit in 128 bytes");
+constexpr uint32_t kPeerMagic = 0x4e42584bu;
 
 }  // namespace
 
@@ -565,6 +633,19 @@ nbody_status nbody_sync(nbody_ctx* c) {
 
 // out[id][3] <- src[i].xyz for the slots [b, e) (src[i] belongs to slot b + i).
 // A host `out` goes through the device staging buffer out3.
+// Peer-exchange mode: copy every rank's owned slice of a per-rank array
+// (acc or cnt, indexed from the owner's first slot) into dst by slot.
+static nbody_status gather_peers(nbody_ctx* c, const void* const* src, void* dst, size_t rec_bytes) {
+  for (int q = 0; q < c->world; ++q) {
+    int64_t b = 0, e = 0;
+    nbody_partition(c->n, q, c->world, &b, &e);
+    if (e > b)
+      CK(cudaMemcpyAsync(static_cast<char*>(dst) + rec_bytes * size_t(b), src[q], rec_bytes * size_t(e - b),
+                         cudaMemcpyDefault, c->stream));
+  }
+  return NBODY_OK;
+}
+
 static nbody_status get_by_id3(nbody_ctx* c, const float4* src, int64_t b, int64_t e, float* out) {
   if (!out) return fail(c, NBODY_EINVAL, "null output");
   const int64_t n = c->n;
@@ -597,6 +678,11 @@ nbody_status nbody_get_accel(nbody_ctx* c, float* out) {
     return get_by_id3(c, c->stage, 0, c->n, out);
   }
 #endif
+  if (c->xpeer) {
+    nbody_status s = gather_peers(c, reinterpret_cast<const void* const*>(c->peer_acc), c->stage, 16);
+    if (s != NBODY_OK) return s;
+    return get_by_id3(c, c->stage, 0, c->n, out);
+  }
   return get_by_id3(c, c->acc, c->own_b, c->own_e, out);
 }
 
@@ -628,6 +714,13 @@ nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
     e = n;
   }
 #endif
+  if (c->xpeer) {
+    nbody_status s = gather_peers(c, reinterpret_cast<const void* const*>(c->peer_cnt), c->stage2, 4);
+    if (s != NBODY_OK) return s;
+    src = c->stage2;
+    b = 0;
+    e = n;
+  }
   const bool dev = is_device_ptr(out);
   uint32_t* dst = dev ? out : reinterpret_cast<uint32_t*>(c->out3);
   if (!dev && (b > 0 || e < n)) CK(cudaMemcpyAsync(dst, out, 4 * size_t(n), cudaMemcpyDefault, c->stream));
@@ -678,6 +771,7 @@ nbody_status nbody_set_partition(nbody_ctx* c, int rank, int world) {
 #ifdef NBODY_WITH_NCCL
   if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is attached");
 #endif
+  if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are attached");
   set_part(c, rank, world);
   drop_graph(c);
   return NBODY_OK;
@@ -740,6 +834,7 @@ nbody_status nbody_attach_nccl(nbody_ctx* c, const void* unique_id, int rank, in
     return fail(c, NBODY_EINVAL, "need a unique id and 0 <= rank < world <= 256");
 #ifdef NBODY_WITH_NCCL
   if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is already attached");
+  if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are attached");
   ncclUniqueId id;
   std::memcpy(&id, unique_id, sizeof(id));
   const ncclResult_t r = ncclCommInitRank(&c->comm, world, id, rank);
@@ -753,6 +848,98 @@ nbody_status nbody_attach_nccl(nbody_ctx* c, const void* unique_id, int rank, in
 #else
   return fail(c, NBODY_ENCCL, "library built without NCCL");
 #endif
+}
+
+// ---- fused exchange over peer memory --------------------------------------
+
+nbody_status nbody_peer_handle(nbody_ctx* c, void* out) {
+  CHECK_CTX(c);
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  PeerDesc d{};
+  CK(cudaIpcGetMemHandle(&d.ipc, c->arena));
+  d.n = c->n;
+  d.arena_bytes = c->arena_bytes;
+  d.magic = kPeerMagic;
+  std::memset(out, 0, 128);
+  std::memcpy(out, &d, sizeof(d));
+  return NBODY_OK;
+}
+
+static nbody_status check_attach(nbody_ctx* c, int rank, int world) {
+  if (world < 1 || world > kMaxPeers || rank < 0 || rank >= world)
+    return fail(c, NBODY_EINVAL, "peer exchange needs 0 <= rank < world <= 8");
+  if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are already attached");
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is attached");
+#endif
+  return NBODY_OK;
+}
+
+nbody_status nbody_attach_peers(nbody_ctx* c, const void* handles, int rank, int world) {
+  CHECK_CTX(c);
+  nbody_status st = check_attach(c, rank, world);
+  if (st != NBODY_OK) return st;
+  if (!handles) return fail(c, NBODY_EINVAL, "null handles");
+  char* base[kMaxPeers] = {};
+  for (int q = 0; q < world; ++q) {
+    PeerDesc d;
+    std::memcpy(&d, static_cast<const char*>(handles) + 128 * size_t(q), sizeof(d));
+    if (d.magic != kPeerMagic || d.n != c->n || d.arena_bytes != c->arena_bytes)
+      return fail(c, NBODY_EINVAL, "peer " + std::to_string(q) + ": descriptor does not match this context");
+    if (q == rank) {
+      base[q] = c->arena;
+      continue;
+    }
+    void* p = nullptr;
+    const cudaError_t e = cudaIpcOpenMemHandle(&p, d.ipc, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      for (int k = 0; k < q; ++k)
+        if (c->peer_map[k]) cudaIpcCloseMemHandle(c->peer_map[k]), c->peer_map[k] = nullptr;
+      return fail(c, NBODY_ECUDA, "cudaIpcOpenMemHandle(peer " + std::to_string(q) + "): " + cudaGetErrorString(e));
+    }
+    c->peer_map[q] = p;
+    base[q] = static_cast<char*>(p);
+  }
+  attach_peer_bases(c, base, rank, world);
+  return NBODY_OK;
+}
+
+nbody_status nbody_attach_peers_local(nbody_ctx** ctxs, int world) {
+  if (!ctxs || world < 1 || world > kMaxPeers) return NBODY_EINVAL;
+  for (int r = 0; r < world; ++r) {
+    nbody_ctx* c = ctxs[r];
+    CHECK_CTX(c);
+    nbody_status st = check_attach(c, r, world);
+    if (st != NBODY_OK) return st;
+    if (c->n != ctxs[0]->n || c->arena_bytes != ctxs[0]->arena_bytes)
+      return fail(c, NBODY_EINVAL, "contexts differ in N");
+  }
+  for (int r = 0; r < world; ++r)  // contexts on different devices: enable peer access
+    for (int q = 0; q < world; ++q) {
+      if (ctxs[r]->device == ctxs[q]->device) continue;
+      nbody_ctx* c = ctxs[r];
+      int prev = -1;
+      CK(cudaGetDevice(&prev));
+      CK(cudaSetDevice(c->device));
+      const cudaError_t e = cudaDeviceEnablePeerAccess(ctxs[q]->device, 0);
+      cudaSetDevice(prev);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+      else if (e != cudaSuccess) return fail(c, NBODY_ECUDA, std::string("peer access: ") + cudaGetErrorString(e));
+    }
+  char* base[kMaxPeers] = {};
+  for (int q = 0; q < world; ++q) base[q] = ctxs[q]->arena;
+  for (int r = 0; r < world; ++r) attach_peer_bases(ctxs[r], base, r, world);
+  return NBODY_OK;
+}
+
+int nbody_exchange_mode(nbody_ctx* c) {
+  if (!c) return -1;
+  if (c->xpeer) return 2;
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) return 1;
+#endif
+  return 0;
 }
 
 nbody_status nbody_get_state(nbody_ctx* c, float* pos_m, float* vel_id) {
@@ -873,6 +1060,8 @@ void nbody_destroy(nbody_ctx* c) {
 #ifdef NBODY_WITH_NCCL
   if (c->comm) ncclCommDestroy(c->comm);
 #endif
+  for (auto& p : c->peer_map)
+    if (p) cudaIpcCloseMemHandle(p);
   if (c->arena) cudaFree(c->arena);
   if (c->quad_arena) cudaFree(c->quad_arena);
   for (auto& e : c->ev)

@@ -116,4 +116,26 @@ void launch_pack_bodies(const float* pos, const float* vel, const float* mass, i
 void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s);
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s);
 
+// ---- K7 fused with the exchange over peer memory -------------
+// Every rank's state buffers and barrier flags, mapped into this process
+// (CUDA IPC over NVLink/NVSwitch, or plain pointers for contexts sharing one
+// device).  Index = rank; the own rank's entries are local pointers.
+constexpr int kMaxPeers = 8;                 // one NVSwitch domain of an HGX B200
+constexpr int kBarrierSlots = 2;             // 0: state consumed, 1: state delivered
+struct PeerTable {
+  float4* pm[kMaxPeers];
+  float4* vi[kMaxPeers];
+  unsigned* flags[kMaxPeers];                // [kBarrierSlots][kMaxPeers] epochs per rank
+  int G = 0, rank = 0;
+};
+// Leapfrog of the owned slots [b, b + len) (acc indexed from 0), storing the
+// new records straight into slot b + i of EVERY rank's pm0/vi0.
+void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t b, int64_t len,
+                             float dt, const PeerTable& pt, cudaStream_t s);
+// Device-side barrier over the G ranks: signal epoch+1 of `slot` to every
+// rank (release, system scope), then wait until every rank's signal for
+// that epoch arrived in the own flag block (acquire).  A wait longer than
+// ~20 s sets *err and returns.
+void launch_xbarrier(const PeerTable& pt, unsigned* epoch, int slot, int* err, cudaStream_t s);
+
 }  // namespace nb

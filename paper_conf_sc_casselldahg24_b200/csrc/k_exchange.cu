@@ -1,0 +1,99 @@
+// k_exchange.cu -- K7 fused with the multi-GPU exchange.
+//
+// Alg. 6 ends every step with the leapfrog update; on G ranks
+// each rank updates only its Hilbert range [A21] and the next step needs the
+// full state on every rank.  Instead of a leapfrog kernel followed by an
+// all-gather, the update kernel stores each new record directly into the
+// same slot of every rank's state buffer (peer memory over NVLink/NVSwitch),
+// so the exchange overlaps the arithmetic store by store.  Two device-side
+// barriers per step order it against the readers:
+//   slot 0  after the permute: every rank has consumed its copy of the old
+//           state, so peers may overwrite it;
+//   slot 1  after the update: every rank's stores have landed.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "internal.cuh"
+
+namespace nb {
+namespace {
+
+__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ uint64_t global_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__global__ __launch_bounds__(256) void k_leapfrog_scatter(const float4* __restrict__ pm_in,
+                                                          const float4* __restrict__ vi_in,
+                                                          const float4* __restrict__ acc, int64_t b, int64_t len,
+                                                          float dt, PeerTable pt) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= len) return;
+  float4 p = pm_in[b + i], v = vi_in[b + i];
+  const float4 a = acc[i];
+  // same operations, same order as k_leapfrog (results bit-identical to G = 1)
+  v.x = fmaf(a.x, dt, v.x);
+  v.y = fmaf(a.y, dt, v.y);
+  v.z = fmaf(a.z, dt, v.z);
+  p.x = fmaf(v.x, dt, p.x);
+  p.y = fmaf(v.y, dt, p.y);
+  p.z = fmaf(v.z, dt, p.z);
+#pragma unroll
+  for (int r = 0; r < kMaxPeers; ++r) {
+    if (r < pt.G) {
+      pt.pm[r][b + i] = p;
+      pt.vi[r][b + i] = v;
+    }
+  }
+}
+
+__global__ void k_xbarrier(PeerTable pt, unsigned* epoch, int slot, int* err) {
+  __shared__ unsigned ep;
+  if (threadIdx.x == 0) {
+    ep = epoch[slot] + 1;
+    epoch[slot] = ep;
+  }
+  __syncthreads();
+  const int q = threadIdx.x;
+  if (q >= pt.G) return;
+  // release: this rank's earlier stores (the previous kernels in stream
+  // order, peer stores included) are visible before the signal
+  __threadfence_system();
+  st_release_sys(pt.flags[q] + slot * kMaxPeers + pt.rank, ep);
+  const unsigned* f = pt.flags[pt.rank] + slot * kMaxPeers + q;
+  if (*reinterpret_cast<volatile int*>(err)) return;  // a peer already timed out: do not hang again
+  const uint64_t t0 = global_ns();
+  while (int(ld_acquire_sys(f) - ep) < 0) {  // epochs only grow (wrap-safe compare)
+    __nanosleep(200);
+    if (global_ns() - t0 > 20ull * 1000000000ull) {
+      atomicExch(err, 1);
+      return;
+    }
+  }
+}
+
+}  // namespace
+
+void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t b, int64_t len,
+                             float dt, const PeerTable& pt, cudaStream_t s) {
+  if (len <= 0) return;
+  k_leapfrog_scatter<<<unsigned((len + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, b, len, dt, pt);
+}
+
+void launch_xbarrier(const PeerTable& pt, unsigned* epoch, int slot, int* err, cudaStream_t s) {
+  k_xbarrier<<<1, 32, 0, s>>>(pt, epoch, slot, err);
+}
+
+}  // namespace nb

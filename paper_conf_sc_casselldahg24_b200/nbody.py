@@ -171,6 +171,40 @@ class NBody:
         from .dist import broadcast_unique_id
         self.attach_nccl(broadcast_unique_id(rank, group), rank, world)
 
+    # fused update + exchange over peer memory (nbody_attach_peers)
+    def peer_handle(self) -> bytes:
+        buf = C.create_string_buffer(128)
+        self._ck(self.lib.nbody_peer_handle(self.h, buf))
+        return buf.raw
+
+    def attach_peers(self, handles, rank: int, world: int):
+        """handles: the world 128-byte descriptors indexed by rank."""
+        blob = b"".join(bytes(h) for h in handles)
+        if len(blob) != 128 * world:
+            raise ValueError("need world descriptors of 128 bytes")
+        buf = C.create_string_buffer(blob, len(blob))
+        self._ck(self.lib.nbody_attach_peers(self.h, buf, int(rank), int(world)))
+
+    def attach_peers_group(self, rank: int, world: int, group=None):
+        """Gather the descriptors over a torch.distributed group and attach."""
+        import torch.distributed as dist
+        handles = [None] * world
+        dist.all_gather_object(handles, self.peer_handle(), group=group)
+        self.attach_peers(handles, rank, world)
+
+    @staticmethod
+    def attach_peers_local(bodies):
+        """Contexts of one process (bodies[r] becomes rank r)."""
+        lib = _capi.load()
+        arr = (C.c_void_p * len(bodies))(*[b.h.value for b in bodies])
+        st = lib.nbody_attach_peers_local(arr, len(bodies))
+        if st != 0:
+            raise _capi.NBodyError(st, "nbody_attach_peers_local: " + "; ".join(
+                lib.nbody_last_error(b.h).decode() for b in bodies if lib.nbody_last_error(b.h)))
+
+    def exchange_mode(self) -> str:
+        return {0: "none", 1: "nccl", 2: "peer"}[self.lib.nbody_exchange_mode(self.h)]
+
     # -- debug views (parity tests) -----------------------------------------
     def debug_keys(self):
         out = np.empty(self.n, np.uint64)

@@ -77,3 +77,139 @@ def test_nccl_world1_matches_plain(NB):
     assert (s.get_positions() == ref.get_positions()).all()
     assert (s.get_accel() == ref.get_accel()).all()
     assert (s.get_interactions() == ref.get_interactions()).all()
+
+
+# ---- fused update + exchange over peer memory (k_exchange.cu) --------------
+
+def _run_peer_local(NB, pos, vel, mass, world, steps, **kw):
+    n = len(pos)
+    ranks = [NB(n, 0.5, 1e-3, 1e-3, **kw) for _ in range(world)]
+    NB.attach_peers_local(ranks)
+    for r, s in enumerate(ranks):
+        assert s.exchange_mode() == "peer"
+        assert s.partition()[:2] == (r, world)
+        s.set_bodies(pos, vel, mass)
+    for _ in range(steps):
+        for s in ranks:  # asynchronous: the device barriers order the ranks
+            s.step(1)
+    for s in ranks:
+        s.sync()
+    return ranks
+
+
+@pytest.mark.parametrize("world,n,kw", [
+    (2, 20_000, {}),
+    (3, 10_007, {}),
+    (8, 40_000, {}),
+    (8, 100, {}),
+    (4, 30_001, {"use_graph": False}),
+    (2, 25_000, {"multipole": 2}),
+    (3, 12_345, {"traversal": 1}),
+])
+def test_peer_exchange_is_bit_identical(NB, world, n, kw):
+    """G contexts on one GPU exchange through k_leapfrog_scatter's stores into
+    every context's state and the device barriers: every rank ends each step
+    with the single-GPU state, bit for bit."""
+    steps = 3
+    pos, vel, mass = generate("plummer", n, 60 + world)
+    ref = NB(n, 0.5, 1e-3, 1e-3, **kw)
+    ref.set_bodies(pos, vel, mass)
+    ref.step(steps)
+    x_ref, v_ref, a_ref = ref.get_positions(), ref.get_velocities(), ref.get_accel()
+    c_ref = ref.get_interactions()
+    ranks = _run_peer_local(NB, pos, vel, mass, world, steps, **kw)
+    total = 0
+    for s in ranks:
+        assert (s.get_positions() == x_ref).all()
+        assert (s.get_velocities() == v_ref).all()
+        assert (s.get_accel() == a_ref).all()          # gathered from the peers
+        assert (s.get_interactions() == c_ref).all()
+        total += s.stats()["interactions"]
+    assert total == ref.stats()["interactions"]
+
+
+def test_peer_exchange_tree_reuse_and_compute_accel(NB):
+    """sort_every = 2 alternates the sorting and the tree-reuse graphs; a
+    compute_accel pass in between keeps the ranks' barrier epochs aligned."""
+    from paper_conf_sc_casselldahg24_b200 import _capi
+    n, world = 16_384, 4
+    pos, vel, mass = generate("disks", n, 71)
+    ref = NB(n, 0.5, 1e-3, 1e-3)
+    ref.set_option(_capi.NBODY_OPT_SORT_EVERY, 2)
+    ref.set_bodies(pos, vel, mass)
+    ref.step(3)
+    ref.compute_accel()
+    ref.step(2)
+    ranks = [NB(n, 0.5, 1e-3, 1e-3) for _ in range(world)]
+    NB.attach_peers_local(ranks)
+    for s in ranks:
+        s.set_option(_capi.NBODY_OPT_SORT_EVERY, 2)
+        s.set_bodies(pos, vel, mass)
+    for k in (3, None, 2):
+        for s in ranks:
+            s.compute_accel() if k is None else s.step(k)
+    for s in ranks:
+        s.sync()
+        assert (s.get_positions() == ref.get_positions()).all()
+        assert (s.get_accel() == ref.get_accel()).all()
+
+
+def test_peer_attach_rejects_mixing(NB):
+    from paper_conf_sc_casselldahg24_b200 import _capi
+    a, b = NB(1000), NB(2000)
+    with pytest.raises(_capi.NBodyError):
+        NB.attach_peers_local([a, b])          # different N
+    c, d = NB(1000), NB(1000)
+    NB.attach_peers_local([c, d])
+    with pytest.raises(_capi.NBodyError):
+        c.set_partition(0, 2)                  # already partitioned by the peers
+    with pytest.raises(_capi.NBodyError):
+        NB.attach_peers_local([c, d])          # twice
+    h = c.peer_handle()
+    assert len(h) == 128
+    e = NB(999)
+    with pytest.raises(_capi.NBodyError):
+        e.attach_peers([h, e.peer_handle()], 1, 2)  # descriptor of another N
+
+
+def _ipc_worker(rank, world, port, n, steps, out_dir):
+    import os
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_casselldahg24_b200 import NBody
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    pos, vel, mass = generate("plummer", n, 90)
+    s = NBody(n, 0.5, 1e-3, 1e-3)
+    s.attach_peers_group(rank, world)
+    s.set_bodies(pos, vel, mass)
+    dist.barrier()
+    s.step(steps)
+    s.sync()
+    np.save(os.path.join(out_dir, f"x{rank}.npy"), s.get_positions())
+    np.save(os.path.join(out_dir, f"a{rank}.npy"), s.get_accel())
+    dist.barrier()
+    s.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.timeout(300)
+def test_peer_exchange_two_processes_ipc(NB, tmp_path):
+    """The multi-process path: two processes (sharing GPU 0) map each other's
+    arena through CUDA IPC, exactly as ranks on different GPUs of one node."""
+    import socket
+    import torch.multiprocessing as mp
+    n, steps, world = 12_000, 3, 2
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    mp.start_processes(_ipc_worker, args=(world, port, n, steps, str(tmp_path)), nprocs=world, join=True,
+                       start_method="spawn")
+    pos, vel, mass = generate("plummer", n, 90)
+    ref = NB(n, 0.5, 1e-3, 1e-3)
+    ref.set_bodies(pos, vel, mass)
+    ref.step(steps)
+    for r in range(world):
+        assert (np.load(tmp_path / f"x{r}.npy") == ref.get_positions()).all()
+        assert (np.load(tmp_path / f"a{r}.npy") == ref.get_accel()).all()
