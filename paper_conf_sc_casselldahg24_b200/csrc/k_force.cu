@@ -316,12 +316,34 @@ constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 constexpr int kCapF = NBODY_CAP_F;  // dense list: entries every active lane interacts with
 constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 
+// Records in pairs, component-interleaved, so that one 16-B shared load
+// yields (x_a, x_b, y_a, y_b) and the interaction of two entries runs on the
+// packed f32x2 pipe (FADD2/FFMA2/FMUL2: half the issue slots, same rounding
+// per element as the scalar instructions).
+struct RecPair {
+  float2 x, y, z, m;
+  __device__ __forceinline__ void put(int h, const float4& r) {
+    reinterpret_cast<float*>(&x)[h] = r.x;
+    reinterpret_cast<float*>(&y)[h] = r.y;
+    reinterpret_cast<float*>(&z)[h] = r.z;
+    reinterpret_cast<float*>(&m)[h] = r.w;
+  }
+  __device__ __forceinline__ float4 get(int h) const {
+    return make_float4(reinterpret_cast<const float*>(&x)[h], reinterpret_cast<const float*>(&y)[h],
+                       reinterpret_cast<const float*>(&z)[h], reinterpret_cast<const float*>(&m)[h]);
+  }
+};
+// Targets in pairs, NEGATED: d = r + (-x) is bit-identical to r - x.
+struct TgtPair {
+  float2 x, y, z, pad;
+};
+
 template <bool kQuad>
 struct V0Smem {
-  float4 tgt[32];        // the warp's target positions
-  float4 frec[kCapF];    // monopole / body records, all lanes
-  float4 prec[kCapP];    // monopole / body records, ...
-  uint32_t pmsk[kCapP];  // ... for the lanes in the mask
+  TgtPair tgt[16];          // the warp's target positions (negated, paired)
+  RecPair frec[kCapF / 2];  // monopole / body records, all lanes
+  RecPair prec[kCapP / 2];  // monopole / body records, ...
+  uint32_t pmsk[kCapP];     // ... for the lanes in the mask
   uint32_t astk[kCapA];
   uint2 tstk[kCapT];     // (id, mask of the targets that reached it)
   uint32_t fid[kQuad ? kCapF : 1];  // NEXT-4: node id of each entry (0: a body)
@@ -355,26 +377,90 @@ __device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const
   if (kQuad && qid) quad_term(a, dx, dy, dz, inv, qf, qid, on);
 }
 
+__device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
+
+// Two monopole interactions on the packed pipe; same per-element operations
+// and order as interact().  (ax, ay, az) hold two partial sums each.
+template <bool kSoft>
+__device__ __forceinline__ void interact2(float2& ax, float2& ay, float2& az, const RecPair& s, float2 m,
+                                          float2 nx, float2 ny, float2 nz, float2 eps2) {
+  const float2 dx = __fadd2_rn(s.x, nx), dy = __fadd2_rn(s.y, ny), dz = __fadd2_rn(s.z, nz);
+  const float2 r2 = __ffma2_rn(dz, dz, __ffma2_rn(dy, dy, __ffma2_rn(dx, dx, eps2)));
+  float2 inv = make_float2(rsqrt_fast(r2.x), rsqrt_fast(r2.y));
+  if (!kSoft) {
+    inv.x = r2.x > 0.f ? inv.x : 0.f;
+    inv.y = r2.y > 0.f ? inv.y : 0.f;
+  }
+  const float2 w = __fmul2_rn(__fmul2_rn(__fmul2_rn(m, inv), inv), inv);
+  ax = __ffma2_rn(w, dx, ax);
+  ay = __ffma2_rn(w, dy, ay);
+  az = __ffma2_rn(w, dz, az);
+}
+
+// Entries [0, cnt) of a pair list; an odd count is padded with a massless
+// entry (it adds exactly 0).
 template <bool kSoft, bool kQuad>
-__device__ __forceinline__ void dense_full(const V0Smem<kQuad>& S, int nf, const Target& T, Acc& a,
-                                           const float4* qf) {
+__device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Target& T, Acc& a, const float4* qf,
+                                           int lane) {
+  if (kQuad) {
 #pragma unroll 4
-  for (int e = 0; e < nf; ++e) {
-    const float4 s = S.frec[e];
-    interact<kSoft, kQuad>(a, s, s.w, T, qf, kQuad ? S.fid[e] : 0u, true);
+    for (int e = 0; e < nf; ++e) {
+      const float4 s = S.frec[e >> 1].get(e & 1);
+      interact<kSoft, kQuad>(a, s, s.w, T, qf, S.fid[e], true);
+    }
+  } else {
+    if (nf & 1) {
+      if (lane == 0) S.frec[nf >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f));
+      __syncwarp();
+    }
+    const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
+    float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
+#pragma unroll 2
+    for (int p = 0; p < (nf + 1) >> 1; ++p) {
+      const RecPair s = S.frec[p];
+      interact2<kSoft>(ax, ay, az, s, s.m, nx, ny, nz, e2);
+    }
+    a.x += ax.x + ax.y;
+    a.y += ay.x + ay.y;
+    a.z += az.x + az.y;
   }
   a.n += uint32_t(nf);
 }
 
 template <bool kSoft, bool kQuad>
-__device__ __forceinline__ void dense_part(const V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane,
+__device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane,
                                            const float4* qf) {
+  if (kQuad) {
 #pragma unroll 4
-  for (int e = 0; e < np; ++e) {
-    const float4 s = S.prec[e];
-    const bool on = (S.pmsk[e] >> lane) & 1u;
-    interact<kSoft, kQuad>(a, s, on ? s.w : 0.f, T, qf, kQuad ? S.pid[e] : 0u, on);
-    a.n += on;
+    for (int e = 0; e < np; ++e) {
+      const float4 s = S.prec[e >> 1].get(e & 1);
+      const bool on = (S.pmsk[e] >> lane) & 1u;
+      interact<kSoft, kQuad>(a, s, on ? s.w : 0.f, T, qf, S.pid[e], on);
+      a.n += on;
+    }
+  } else {
+    if (np & 1) {
+      if (lane == 0) {
+        S.prec[np >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f));
+        S.pmsk[np] = 0u;
+      }
+      __syncwarp();
+    }
+    const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
+    float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
+    uint32_t cnt = 0;
+#pragma unroll 2
+    for (int p = 0; p < (np + 1) >> 1; ++p) {
+      const RecPair s = S.prec[p];
+      const uint2 mk = *reinterpret_cast<const uint2*>(&S.pmsk[2 * p]);
+      const bool on0 = (mk.x >> lane) & 1u, on1 = (mk.y >> lane) & 1u;
+      interact2<kSoft>(ax, ay, az, s, make_float2(on0 ? s.m.x : 0.f, on1 ? s.m.y : 0.f), nx, ny, nz, e2);
+      cnt += uint32_t(on0) + uint32_t(on1);
+    }
+    a.x += ax.x + ax.y;
+    a.y += ay.x + ay.y;
+    a.z += az.x + az.y;
+    a.n += cnt;
   }
 }
 
@@ -398,7 +484,12 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   const int L = W.L;
   const uint32_t kid = leaf0 + uint32_t(k);
   const uint32_t kid0 = leaf0 + uint32_t(k0);
-  S.tgt[lane] = make_float4(T.x, T.y, T.z, 0.f);
+  {
+    TgtPair& tp = S.tgt[lane >> 1];
+    reinterpret_cast<float*>(&tp.x)[lane & 1] = -T.x;
+    reinterpret_cast<float*>(&tp.y)[lane & 1] = -T.y;
+    reinterpret_cast<float*>(&tp.z)[lane & 1] = -T.z;
+  }
 
   // group box over the active lanes (exact fp32 min/max, used in fp64)
   const float inf = __int_as_float(0x7f800000);
@@ -420,12 +511,12 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
     const uint32_t bp = __ballot_sync(kFull, part);
     if (full) {
       const int pos = nf + __popc(bf & lt);
-      S.frec[pos] = r;
+      S.frec[pos >> 1].put(pos & 1, r);
       if (kQuad) S.fid[pos] = id;
     }
     if (part) {
       const int pos = np + __popc(bp & lt);
-      S.prec[pos] = r;
+      S.prec[pos >> 1].put(pos & 1, r);
       S.pmsk[pos] = msk;
       if (kQuad) S.pid[pos] = id;
     }
@@ -435,7 +526,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   auto flush = [&](bool all) {
     __syncwarp();
     if (nf > kCapF - 32 || (all && nf > 0)) {
-      dense_full<kSoft, kQuad>(S, nf, T, a, qf);
+      dense_full<kSoft, kQuad>(S, nf, T, a, qf, lane);
       nf = 0;
     }
     if (np > kCapP - 32 || (all && np > 0)) {
@@ -458,13 +549,16 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       const float4 r = __ldg(W.rec + g);
       const float2 c = __ldg(W.rc + g);  // leaves: (-inf, -inf): always interact
       uint32_t am = 0u, rm = 0u;
+      {
+        const float2 rx = f2(r.x), ry = f2(r.y), rz = f2(r.z);
 #pragma unroll
-      for (int t = 0; t < 32; ++t) {
-        const float4 tp = S.tgt[t];
-        const float dx = r.x - tp.x, dy = r.y - tp.y, dz = r.z - tp.z;
-        const float d2 = fmaf(dz, dz, fmaf(dy, dy, dx * dx));
-        am |= d2 > c.y ? (1u << t) : 0u;
-        rm |= d2 < c.x ? (1u << t) : 0u;
+        for (int t = 0; t < 16; ++t) {  // two targets per packed operation
+          const TgtPair tp = S.tgt[t];
+          const float2 dx = __fadd2_rn(rx, tp.x), dy = __fadd2_rn(ry, tp.y), dz = __fadd2_rn(rz, tp.z);
+          const float2 d2 = __ffma2_rn(dz, dz, __ffma2_rn(dy, dy, __fmul2_rn(dx, dx)));
+          am |= (d2.x > c.y ? (1u << (2 * t)) : 0u) | (d2.y > c.y ? (2u << (2 * t)) : 0u);
+          rm |= (d2.x < c.x ? (1u << (2 * t)) : 0u) | (d2.y < c.x ? (2u << (2 * t)) : 0u);
+        }
       }
       am &= m;
       rm &= m;
@@ -474,8 +568,11 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
           const double4 pd = W.pred[g];
           do {
             const int t = __ffs(int(und)) - 1;
-            const float4 tp = S.tgt[t];
-            if (opening_accept64(pd, tp.x, tp.y, tp.z, T.th2)) am |= 1u << t; else rm |= 1u << t;
+            const TgtPair& tp = S.tgt[t >> 1];
+            const float x = -reinterpret_cast<const float*>(&tp.x)[t & 1];
+            const float y = -reinterpret_cast<const float*>(&tp.y)[t & 1];
+            const float z = -reinterpret_cast<const float*>(&tp.z)[t & 1];
+            if (opening_accept64(pd, x, y, z, T.th2)) am |= 1u << t; else rm |= 1u << t;
             und &= und - 1u;
           } while (und);
         }
