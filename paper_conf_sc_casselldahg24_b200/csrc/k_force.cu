@@ -320,7 +320,7 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 // yields (x_a, x_b, y_a, y_b) and the interaction of two entries runs on the
 // packed f32x2 pipe (FADD2/FFMA2/FMUL2: half the issue slots, same rounding
 // per element as the scalar instructions).
-struct RecPair {
+struct alignas(16) RecPair {
   float2 x, y, z, m;
   __device__ __forceinline__ void put(int h, const float4& r) {
     reinterpret_cast<float*>(&x)[h] = r.x;
@@ -334,12 +334,12 @@ struct RecPair {
   }
 };
 // Targets in pairs, NEGATED: d = r + (-x) is bit-identical to r - x.
-struct TgtPair {
+struct alignas(16) TgtPair {
   float2 x, y, z, pad;
 };
 
 template <bool kQuad>
-struct V0Smem {
+struct alignas(16) V0Smem {
   TgtPair tgt[16];          // the warp's target positions (negated, paired)
   RecPair frec[kCapF / 2];  // monopole / body records, all lanes
   RecPair prec[kCapP / 2];  // monopole / body records, ...
@@ -550,14 +550,25 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       const float2 c = __ldg(W.rc + g);  // leaves: (-inf, -inf): always interact
       uint32_t am = 0u, rm = 0u;
       {
+        // d2 > hi  <=>  hi - d2 < 0 and d2 < lo  <=>  d2 - lo < 0: one exact
+        // rounding each (a nonzero difference keeps its sign; x - x = +0;
+        // -inf thresholds give -inf / +inf), so the sign bits are the
+        // comparisons, shifted into the masks from bit 31 down.
         const float2 rx = f2(r.x), ry = f2(r.y), rz = f2(r.z);
+        const float2 hi = f2(c.y), nlo = f2(-c.x), m1 = f2(-1.f);
 #pragma unroll
-        for (int t = 0; t < 16; ++t) {  // two targets per packed operation
-          const TgtPair tp = S.tgt[t];
-          const float2 dx = __fadd2_rn(rx, tp.x), dy = __fadd2_rn(ry, tp.y), dz = __fadd2_rn(rz, tp.z);
+        for (int t = 15; t >= 0; --t) {  // two targets per packed operation
+          const float4 xy = *reinterpret_cast<const float4*>(&S.tgt[t].x);
+          const float2 tz = S.tgt[t].z;
+          const float2 dx = __fadd2_rn(rx, make_float2(xy.x, xy.y)), dy = __fadd2_rn(ry, make_float2(xy.z, xy.w)),
+                       dz = __fadd2_rn(rz, tz);
           const float2 d2 = __ffma2_rn(dz, dz, __ffma2_rn(dy, dy, __fmul2_rn(dx, dx)));
-          am |= (d2.x > c.y ? (1u << (2 * t)) : 0u) | (d2.y > c.y ? (2u << (2 * t)) : 0u);
-          rm |= (d2.x < c.x ? (1u << (2 * t)) : 0u) | (d2.y < c.x ? (2u << (2 * t)) : 0u);
+          const float2 sa = __ffma2_rn(d2, m1, hi);   // hi - d2
+          const float2 sr = __fadd2_rn(d2, nlo);      // d2 - lo
+          am = __funnelshift_l(__float_as_uint(sa.y), am, 1);
+          am = __funnelshift_l(__float_as_uint(sa.x), am, 1);
+          rm = __funnelshift_l(__float_as_uint(sr.y), rm, 1);
+          rm = __funnelshift_l(__float_as_uint(sr.x), rm, 1);
         }
       }
       am &= m;
