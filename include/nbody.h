@@ -248,6 +248,12 @@ nbody_status nbody_debug_level(nbody_ctx *ctx, int level, int64_t *count, double
  * (xx, yy, zz, xy, xz, yz) [A24]. */
 nbody_status nbody_debug_quad(nbody_ctx *ctx, int level, double *S);
 
+/* Design instrumentation of K6: copies up to n event counters of the
+ * traversal (summed over all force passes since the last call, then reset)
+ * into out and returns how many were written; 0 unless the library was built
+ * with -DNBODY_K6_STATS (never in the product build). */
+int nbody_debug_force_stats(uint64_t *out, int n);
+
 /* Human-readable description of the last error on this context (never NULL). */
 const char *nbody_last_error(const nbody_ctx *ctx);
 

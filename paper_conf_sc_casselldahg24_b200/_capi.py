@@ -52,6 +52,7 @@ _S = C.c_int
 SIGNATURES = {
     "nbody_version": (C.c_int, []),
     "nbody_select_device": (_S, [C.c_int]),
+    "nbody_debug_force_stats": (C.c_int, [_P, C.c_int]),
     "nbody_create": (_S, [_I64, C.c_double, C.c_double, C.c_double, C.POINTER(_P)]),
     "nbody_set_option": (_S, [_P, C.c_int, _I64]),
     "nbody_set_bodies": (_S, [_P, _P, _P, _P]),

@@ -1020,6 +1020,11 @@ nbody_status nbody_debug_perm(nbody_ctx* c, uint32_t* perm) {
   return sync_stream(c);
 }
 
+int nbody_debug_force_stats(uint64_t* out, int n) {
+  if (!out || n <= 0) return 0;
+  return force_stats(reinterpret_cast<unsigned long long*>(out), n);
+}
+
 nbody_status nbody_debug_quad(nbody_ctx* c, int level, double* S) {
   CHECK_CTX(c);
   if (level < 1 || level > c->tree.L) return fail(c, NBODY_EINVAL, "level out of range [1, L]");

@@ -100,6 +100,9 @@ void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, 
 
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
+// K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
+constexpr int kK6Stats = 16;
+int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
 int64_t direct_chunks(int64_t n, int64_t nt);

@@ -51,6 +51,31 @@
 #include "internal.cuh"
 
 namespace nb {
+
+// Traversal event counters for design work (NBODY_K6_STATS builds only;
+// read with nbody_debug_force_stats).  Index meaning: see kStatNames in
+// scripts/k6_stats.py.
+#ifdef NBODY_K6_STATS
+__device__ unsigned long long g_k6_stats[kK6Stats];
+#define K6STAT(i, v) (st[i] += (v))
+#else
+#define K6STAT(i, v) ((void)0)
+#endif
+
+int force_stats(unsigned long long* out, int n) {
+#ifdef NBODY_K6_STATS
+  if (n > kK6Stats) n = kK6Stats;
+  if (cudaMemcpyFromSymbol(out, g_k6_stats, sizeof(unsigned long long) * n) != cudaSuccess) return -1;
+  static const unsigned long long zero[kK6Stats] = {};
+  if (cudaMemcpyToSymbol(g_k6_stats, zero, sizeof(zero)) != cudaSuccess) return -1;
+  return n;
+#else
+  (void)out;
+  (void)n;
+  return 0;
+#endif
+}
+
 namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
@@ -498,6 +523,10 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   const float blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
 
   int na = 1, nt = 0, nf = 0, np = 0;
+#ifdef NBODY_K6_STATS
+  unsigned long long st[kK6Stats] = {};
+#endif
+  K6STAT(0, 1);
   if (lane == 0) S.astk[0] = 1u;
   __syncwarp();
 
@@ -522,15 +551,23 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
     }
     nf += __popc(bf);
     np += __popc(bp);
+    K6STAT(5, __popc(bf));
+    K6STAT(6, __popc(bp));
+    K6STAT(7, __reduce_add_sync(kFull, part ? __popc(msk) : 0u));
+    K6STAT(8, __popc(bf) * __popc(amask));
   };
   auto flush = [&](bool all) {
     __syncwarp();
     if (nf > kCapF - 32 || (all && nf > 0)) {
       dense_full<kSoft, kQuad>(S, nf, T, a, qf, lane);
+      K6STAT(10, 1);
+      K6STAT(11, (nf + 1) >> 1);
       nf = 0;
     }
     if (np > kCapP - 32 || (all && np > 0)) {
       dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
+      K6STAT(12, 1);
+      K6STAT(13, (np + 1) >> 1);
       np = 0;
     }
     __syncwarp();
@@ -541,6 +578,9 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       // ---- T: transposed classification of up to 32 (node, mask) entries
       const int take = nt < 32 ? nt : 32;
       const int base = nt - take;
+      K6STAT(3, 1);
+      K6STAT(4, take);
+      K6STAT(15, take < 32);
       const bool has = lane < take;
       const uint2 e = has ? S.tstk[base + lane] : make_uint2(leaf0, 0u);
       __syncwarp();
@@ -574,6 +614,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       am &= m;
       rm &= m;
       uint32_t und = m & ~(am | rm);
+      K6STAT(9, __reduce_add_sync(kFull, __popc(und)));
       if (__any_sync(kFull, und != 0u)) {  // rare: exact fp64 decisions
         if (und) {
           const double4 pd = W.pred[g];
@@ -608,6 +649,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       uint32_t spill = __ballot_sync(kFull, rm != 0u && !room);
       while (spill) {
         const int src = __ffs(int(spill)) - 1;
+        K6STAT(14, 1);
         spill &= spill - 1u;
         const uint32_t gs = __shfl_sync(kFull, g, src);
         const uint32_t ms = __shfl_sync(kFull, rm, src);
@@ -619,6 +661,8 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       // ---- A: box classification of up to 32 nodes reached by every lane
       const int take = na < 32 ? na : 32;
       const int base = na - take;
+      K6STAT(1, 1);
+      K6STAT(2, take);
       const bool has = lane < take;
       const uint32_t g = has ? S.astk[base + lane] : 0u;
       __syncwarp();
@@ -681,6 +725,10 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   }
   flush(true);
   store_result(P, k, active, a, lane);
+#ifdef NBODY_K6_STATS
+  if (lane == 0)
+    for (int i = 0; i < kK6Stats; ++i) atomicAdd(&g_k6_stats[i], st[i]);
+#endif
 }
 
 }  // namespace
