@@ -212,6 +212,7 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 16 * size_t(inner);                     // blo
   sz[k++] = 16 * size_t(inner);                     // bhi
   sz[k++] = 8 * size_t(ids);                        // rc (-inf at the leaves)
+  sz[k++] = 16 * size_t(inner);                     // tf
   sz[k++] = 256;                                    // exchange flags, epochs, error
   size_t total = 0;
   for (int i = 0; i < k; ++i) total += align_up(sz[i]);
@@ -248,6 +249,7 @@ nbody_status allocate(nbody_ctx* c) {
   c->tree.blo = (float4*)take();
   c->tree.bhi = (float4*)take();
   c->tree.rc = (float2*)take();
+  c->tree.tf = (float4*)take();
   c->xflags = (unsigned*)take();
   c->xepoch = c->xflags + kBarrierSlots * kMaxPeers;
   c->xerr = reinterpret_cast<int*>(c->xepoch + kBarrierSlots);

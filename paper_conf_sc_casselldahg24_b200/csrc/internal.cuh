@@ -21,6 +21,7 @@ struct GridInfo {
   int b;         // bits per axis
   float abs_d2;  // absolute slack of the fp32 opening-test filter: 1e-9 R^2,
                  // R = max |coordinate| (K6)
+  float R;       // max |coordinate| of this step's bodies (T-filter slack)
 };
 
 // NEXT-4 [A24]: second mass moment about the COM, S = sum m (x-c)(x-c)^T.
@@ -41,6 +42,8 @@ struct TreeView {
                    // opening test: d2 < lo => open, d2 > hi => accept, else
                    // the exact fp64 test; leaves
                    // hold (-inf, -inf)
+  float4* tf;      // internal ids: (fl32(com64 - c32) x, y, z, fl32(s^2 / th2)):
+                   // the T-phase filter data (k_force.cu tfilter_prep)
   const GridInfo* grid;  // bbox of this step (filter slack)
   double th2;            // theta^2 the thresholds were built for
   double4* mom;    // (M, Mx, My, Mz) fp64 moments (build only) [A12]
@@ -101,7 +104,7 @@ void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, 
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
-constexpr int kK6Stats = 16;
+constexpr int kK6Stats = 32;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------

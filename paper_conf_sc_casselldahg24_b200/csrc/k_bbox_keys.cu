@@ -82,6 +82,7 @@ __global__ void k_bbox_final(const float* __restrict__ partial, int nparts, int 
     float R = 0.f;
     for (int k = 0; k < 6; ++k) R = fmaxf(R, fabsf(s[k]));
     g->abs_d2 = fmaxf(1e-9f * R * R, 1e-37f);  // larger slack only sends more decisions to fp64
+    g->R = R;
   }
 }
 

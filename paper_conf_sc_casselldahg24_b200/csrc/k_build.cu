@@ -69,8 +69,14 @@ __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, dou
     rc.x = rc.y = __int_as_float(0x7f800000);
   }
   t.rc[node] = rc;
-  t.rec[node] =
-      make_float4(__double2float_rn(c[0]), __double2float_rn(c[1]), __double2float_rn(c[2]), __double2float_rn(M));
+  const float c0 = __double2float_rn(c[0]), c1 = __double2float_rn(c[1]), c2 = __double2float_rn(c[2]);
+  t.rec[node] = make_float4(c0, c1, c2, __double2float_rn(M));
+  // T-phase filter data: the fp32 residuals of the COM (com64 - c32 is exact
+  // in fp64) and q = s^2 / theta^2 (+inf at theta = 0)
+  t.tf[node] = make_float4(__double2float_rn(__dsub_rn(c[0], double(c0))),
+                           __double2float_rn(__dsub_rn(c[1], double(c1))),
+                           __double2float_rn(__dsub_rn(c[2], double(c2))),
+                           t.th2 > 0.0 ? __double2float_rn(__ddiv_rn(s2, t.th2)) : __int_as_float(0x7f800000));
   if (S) {
     if (keep) {
 #pragma unroll

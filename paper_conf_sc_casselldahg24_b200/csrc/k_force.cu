@@ -325,7 +325,7 @@ constexpr int kV0Warps = 4;
 // stack overflow is handled (box phase: hand over as MIXED; transposed
 // phase: per-lane mask walk), so the capacities only affect speed.
 #ifndef NBODY_CAP_T
-#define NBODY_CAP_T 352
+#define NBODY_CAP_T 288
 #endif
 #ifndef NBODY_V0_MINB
 #define NBODY_V0_MINB 8
@@ -358,14 +358,16 @@ struct alignas(16) RecPair {
                        reinterpret_cast<const float*>(&z)[h], reinterpret_cast<const float*>(&m)[h]);
   }
 };
-// Targets in pairs, NEGATED: d = r + (-x) is bit-identical to r - x.
+// Targets in pairs for the transposed test, relative to the group reference
+// point g: p = 2 x', q = -|x'|^2 with x' = fl(x - g) (see tfilter_prep).
 struct alignas(16) TgtPair {
-  float2 x, y, z, pad;
+  float2 px, py, pz, q;
 };
 
 template <bool kQuad>
 struct alignas(16) V0Smem {
-  TgtPair tgt[16];          // the warp's target positions (negated, paired)
+  TgtPair tgt[16];          // the warp's targets for the transposed test (paired)
+  float4 tpos[32];          // the warp's target positions (fp64 fallback)
   RecPair frec[kCapF / 2];  // monopole / body records, all lanes
   RecPair prec[kCapP / 2];  // monopole / body records, ...
   uint32_t pmsk[kCapP];     // ... for the lanes in the mask
@@ -404,6 +406,38 @@ __device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const
 
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 
+// Transposed-phase filter of the fp64 opening test.
+// With g the group reference point (fp32), c~ = com64 - g, x~ = x - g (exact
+// reals): D^2 = |com64 - x|^2 = |c~|^2 - S*,  S* = 2 c~.x~ - |x~|^2.  Each
+// target evaluates S = fma(2x'_x, c'_x, fma(2x'_y, c'_y, fma(2x'_z, c'_z, q)))
+// in fp32 from x' = fl(x - g), q = fl(-|x'|^2) and the node's
+// c' = fl(fl(c32 - g) + lo), lo = fl32(com64 - c32) (tf).  With b >= |x~|,
+// R >= every |coordinate| and L1 = |c'|_1:
+//   |c' - c~|_i <= 2.01u |c~_i| + 4u^2 R,  |S - S*| <= u b (12.2 L1 + 6.2 b + 24u R),
+//   | fl(|c'|^2) - |c~|^2 | <= 7.1u a2 + 8u^2 R L1          (u = 2^-24),
+// so with E2 = u ((13 b + 5e-7 R) L1 + 7 b^2 + 2e-6 b R) (kk1 = 13 b + 5e-7 R,
+// kk0 = 7 b^2 + 2e-6 b R, per warp) and q32 = fl32(s^2/th2) (error <= 1.01u):
+//   S < KA = a2 (1 - 8u) - q32 (1 + 2u) - E2  (rounded down)  =>  D^2 > q (1 + 2e-15)
+//        => the fp64 test accepts;
+//   S > KO = a2 (1 + 8u) - q32 (1 - 2u) + E2  (rounded up)    =>  D^2 < q (1 - 2e-15)
+//        => it opens;
+// otherwise (or NaN) the exact fp64 test decides.  theta = 0: q32 = +inf, so
+// KA = KO = -inf (everything opens).
+__device__ __forceinline__ void tfilter_prep(const float4& r, const float4& tf, float gx, float gy, float gz,
+                                             float kk1, float kk0, float& cx, float& cy, float& cz, float& KA,
+                                             float& KO) {
+  cx = (r.x - gx) + tf.x;
+  cy = (r.y - gy) + tf.y;
+  cz = (r.z - gz) + tf.z;
+  const float L1 = __fadd_ru(__fadd_ru(fabsf(cx), fabsf(cy)), fabsf(cz));
+  const float E2 = __fmul_ru(__fmaf_ru(kk1, L1, kk0), 5.9604644775390625e-08f);
+  const float a2 = fmaf(cz, cz, fmaf(cy, cy, cx * cx));
+  constexpr float kU8m = 1.f - 8.f * 5.9604644775390625e-08f, kU8p = 1.f + 8.f * 5.9604644775390625e-08f;
+  constexpr float kU2m = 1.f - 2.f * 5.9604644775390625e-08f, kU2p = 1.f + 2.f * 5.9604644775390625e-08f;
+  KA = __fsub_rd(__fsub_rd(__fmul_rd(a2, kU8m), __fmul_ru(tf.w, kU2p)), E2);
+  KO = __fadd_ru(__fsub_ru(__fmul_ru(a2, kU8p), __fmul_rd(tf.w, kU2m)), E2);
+}
+
 // Two monopole interactions on the packed pipe; same per-element operations
 // and order as interact().  (ax, ay, az) hold two partial sums each.
 template <bool kSoft>
@@ -416,7 +450,7 @@ __device__ __forceinline__ void interact2(float2& ax, float2& ay, float2& az, co
     inv.x = r2.x > 0.f ? inv.x : 0.f;
     inv.y = r2.y > 0.f ? inv.y : 0.f;
   }
-  const float2 w = __fmul2_rn(__fmul2_rn(__fmul2_rn(m, inv), inv), inv);
+  const float2 w = __fmul2_rn(__fmul2_rn(m, inv), __fmul2_rn(inv, inv));  // m inv^3, two-deep
   ax = __ffma2_rn(w, dx, ax);
   ay = __ffma2_rn(w, dy, ay);
   az = __ffma2_rn(w, dz, az);
@@ -504,27 +538,41 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   Acc a;
   const uint32_t lt = (1u << lane) - 1u;
   const Walk W = make_walk(P);
+  const float4* tfp = in_reg(P.t.tf);
   const uint32_t leaf0 = W.leaf0;
   const uint32_t n = W.n;
   const int L = W.L;
   const uint32_t kid = leaf0 + uint32_t(k);
   const uint32_t kid0 = leaf0 + uint32_t(k0);
-  {
-    TgtPair& tp = S.tgt[lane >> 1];
-    reinterpret_cast<float*>(&tp.x)[lane & 1] = -T.x;
-    reinterpret_cast<float*>(&tp.y)[lane & 1] = -T.y;
-    reinterpret_cast<float*>(&tp.z)[lane & 1] = -T.z;
-  }
-
   // group box over the active lanes (exact fp32 min/max, used in fp64)
   const float inf = __int_as_float(0x7f800000);
   const float blx = warp_minf(active ? T.x : inf), bhx = warp_maxf(active ? T.x : -inf);
   const float bly = warp_minf(active ? T.y : inf), bhy = warp_maxf(active ? T.y : -inf);
   const float blz = warp_minf(active ? T.z : inf), bhz = warp_maxf(active ? T.z : -inf);
+  // transposed-test frame: reference g = box midpoint, x' = fl(x - g), and
+  // bR >= |x - g| for every target (tfilter_prep)
+  const float gx = 0.5f * blx + 0.5f * bhx, gy = 0.5f * bly + 0.5f * bhy, gz = 0.5f * blz + 0.5f * bhz;
+  float kk1, kk0;
+  {
+    const float ux = active ? T.x - gx : 0.f, uy = active ? T.y - gy : 0.f, uz = active ? T.z - gz : 0.f;
+    const double u2 = fma(double(uz), double(uz), fma(double(uy), double(uy), double(ux) * double(ux)));
+    TgtPair& tp = S.tgt[lane >> 1];
+    reinterpret_cast<float*>(&tp.px)[lane & 1] = 2.f * ux;
+    reinterpret_cast<float*>(&tp.py)[lane & 1] = 2.f * uy;
+    reinterpret_cast<float*>(&tp.pz)[lane & 1] = 2.f * uz;
+    reinterpret_cast<float*>(&tp.q)[lane & 1] = float(-u2);
+    S.tpos[lane] = make_float4(T.x, T.y, T.z, 0.f);
+    // b >= |x - g| = |x'| (1 + O(u)): 4e-7 > 2u + rounding of the bound
+    const float b = __fmul_ru(warp_maxf(__fsqrt_ru(__double2float_ru(u2))), 1.f + 4e-7f);
+    const float R = P.grid->R;
+    kk1 = __fmaf_ru(13.f, b, __fmul_ru(5e-7f, R));
+    kk0 = __fmaf_ru(__fmul_ru(7.f, b), b, __fmul_ru(__fmul_ru(2e-6f, b), R));
+  }
 
   int na = 1, nt = 0, nf = 0, np = 0;
 #ifdef NBODY_K6_STATS
   unsigned long long st[kK6Stats] = {};
+  int sq[4] = {0, 0, 0, 0}, sh[2] = {0, 0}, s8[8] = {}, s16[16] = {}, s32 = 0;
 #endif
   K6STAT(0, 1);
   if (lane == 0) S.astk[0] = 1u;
@@ -555,6 +603,29 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
     K6STAT(6, __popc(bp));
     K6STAT(7, __reduce_add_sync(kFull, part ? __popc(msk) : 0u));
     K6STAT(8, __popc(bf) * __popc(amask));
+#ifdef NBODY_K6_STATS
+    {
+      const uint32_t q0 = __ballot_sync(kFull, part && (msk & 0xffu)), q1 = __ballot_sync(kFull, part && (msk & 0xff00u));
+      const uint32_t q2 = __ballot_sync(kFull, part && (msk & 0xff0000u)),
+                     q3 = __ballot_sync(kFull, part && (msk & 0xff000000u));
+      const uint32_t h0 = __ballot_sync(kFull, part && (msk & 0xffffu)), h1 = __ballot_sync(kFull, part && (msk >> 16));
+      const int nq = __popc(q0) + __popc(q1) + __popc(q2) + __popc(q3);
+      K6STAT(19, nq);
+      K6STAT(20, __reduce_add_sync(kFull, part && (((msk & 0xffu) == msk) || ((msk & 0xff00u) == msk) ||
+                                                     ((msk & 0xff0000u) == msk) || ((msk & 0xff000000u) == msk))));
+      K6STAT(21, __popc(h0) + __popc(h1));
+      sq[0] += __popc(q0); sq[1] += __popc(q1); sq[2] += __popc(q2); sq[3] += __popc(q3);
+      sh[0] += __popc(h0); sh[1] += __popc(h1);
+      for (int j = 0; j < 8; ++j) s8[j] += __popc(__ballot_sync(kFull, part && ((msk >> (4 * j)) & 0xfu)));
+      for (int j = 0; j < 16; ++j) s16[j] += __popc(__ballot_sync(kFull, part && ((msk >> (2 * j)) & 0x3u)));
+      s32 += part ? 0 : 0;
+      for (int j = 0; j < 32; ++j) {
+        const uint32_t mj = __shfl_sync(kFull, msk, j);
+        const bool pj = __shfl_sync(kFull, part, j);
+        s32 += pj && ((mj >> lane) & 1u);
+      }
+    }
+#endif
   };
   auto flush = [&](bool all) {
     __syncwarp();
@@ -568,6 +639,20 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
       K6STAT(12, 1);
       K6STAT(13, (np + 1) >> 1);
+#ifdef NBODY_K6_STATS
+      K6STAT(22, max(max(sq[0], sq[1]), max(sq[2], sq[3])));
+      K6STAT(23, max(sh[0], sh[1]));
+      sq[0] = sq[1] = sq[2] = sq[3] = sh[0] = sh[1] = 0;
+      {
+        int m8 = 0, m16 = 0;
+        for (int j = 0; j < 8; ++j) { m8 = max(m8, s8[j]); s8[j] = 0; }
+        for (int j = 0; j < 16; ++j) { m16 = max(m16, s16[j]); s16[j] = 0; }
+        K6STAT(26, m8);
+        K6STAT(27, m16);
+        K6STAT(28, __reduce_max_sync(kFull, uint32_t(s32)));
+        s32 = 0;
+      }
+#endif
       np = 0;
     }
     __syncwarp();
@@ -587,24 +672,27 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       nt = base;
       const uint32_t g = e.x, m = e.y;
       const float4 r = __ldg(W.rec + g);
-      const float2 c = __ldg(W.rc + g);  // leaves: (-inf, -inf): always interact
+      float cx = 0.f, cy = 0.f, cz = 0.f;
+      float KA = inf, KO = inf;  // leaves: always interact, never open
+      if (g < leaf0) tfilter_prep(r, __ldg(tfp + g), gx, gy, gz, kk1, kk0, cx, cy, cz, KA, KO);
       uint32_t am = 0u, rm = 0u;
       {
-        // d2 > hi  <=>  hi - d2 < 0 and d2 < lo  <=>  d2 - lo < 0: one exact
-        // rounding each (a nonzero difference keeps its sign; x - x = +0;
-        // -inf thresholds give -inf / +inf), so the sign bits are the
+        // S = 2 c'.x' - |x'|^2; accept iff S < KA  <=>  S - KA < 0, open iff
+        // S > KO  <=>  KO - S < 0: one exact rounding each (a nonzero
+        // difference keeps its sign; x - x = +0; infinite thresholds give
+        // infinities of the right sign), so the sign bits are the
         // comparisons, shifted into the masks from bit 31 down.
-        const float2 rx = f2(r.x), ry = f2(r.y), rz = f2(r.z);
-        const float2 hi = f2(c.y), nlo = f2(-c.x), m1 = f2(-1.f);
+        const float2 nKA = f2(-KA), vKO = f2(KO), m1 = f2(-1.f);
 #pragma unroll
         for (int t = 15; t >= 0; --t) {  // two targets per packed operation
-          const float4 xy = *reinterpret_cast<const float4*>(&S.tgt[t].x);
-          const float2 tz = S.tgt[t].z;
-          const float2 dx = __fadd2_rn(rx, make_float2(xy.x, xy.y)), dy = __fadd2_rn(ry, make_float2(xy.z, xy.w)),
-                       dz = __fadd2_rn(rz, tz);
-          const float2 d2 = __ffma2_rn(dz, dz, __ffma2_rn(dy, dy, __fmul2_rn(dx, dx)));
-          const float2 sa = __ffma2_rn(d2, m1, hi);   // hi - d2
-          const float2 sr = __fadd2_rn(d2, nlo);      // d2 - lo
+          const float4 pxy = *reinterpret_cast<const float4*>(&S.tgt[t].px);
+          const float4 pzq = *reinterpret_cast<const float4*>(&S.tgt[t].pz);
+          const float2 sv = __ffma2_rn(make_float2(pxy.x, pxy.y), f2(cx),
+                                       __ffma2_rn(make_float2(pxy.z, pxy.w), f2(cy),
+                                                  __ffma2_rn(make_float2(pzq.x, pzq.y), f2(cz),
+                                                             make_float2(pzq.z, pzq.w))));
+          const float2 sa = __fadd2_rn(sv, nKA);      // S - KA
+          const float2 sr = __ffma2_rn(sv, m1, vKO);  // KO - S
           am = __funnelshift_l(__float_as_uint(sa.y), am, 1);
           am = __funnelshift_l(__float_as_uint(sa.x), am, 1);
           rm = __funnelshift_l(__float_as_uint(sr.y), rm, 1);
@@ -615,16 +703,19 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       rm &= m;
       uint32_t und = m & ~(am | rm);
       K6STAT(9, __reduce_add_sync(kFull, __popc(und)));
+      K6STAT(16, __reduce_add_sync(kFull, has && (((m & 0xffu) == m) || ((m & 0xff00u) == m) ||
+                                                  ((m & 0xff0000u) == m) || ((m & 0xff000000u) == m))));
+      K6STAT(17, __reduce_add_sync(kFull, has && (((m & 0xffffu) == m) || ((m >> 16) << 16) == m)));
+      K6STAT(18, __reduce_add_sync(kFull, has ? __popc(m) : 0u));
+      K6STAT(24, __reduce_add_sync(kFull, has ? __popc(am) : 0u));
+      K6STAT(25, __reduce_add_sync(kFull, has ? __popc(rm) : 0u));
       if (__any_sync(kFull, und != 0u)) {  // rare: exact fp64 decisions
         if (und) {
           const double4 pd = W.pred[g];
           do {
             const int t = __ffs(int(und)) - 1;
-            const TgtPair& tp = S.tgt[t >> 1];
-            const float x = -reinterpret_cast<const float*>(&tp.x)[t & 1];
-            const float y = -reinterpret_cast<const float*>(&tp.y)[t & 1];
-            const float z = -reinterpret_cast<const float*>(&tp.z)[t & 1];
-            if (opening_accept64(pd, x, y, z, T.th2)) am |= 1u << t; else rm |= 1u << t;
+            const float4 tp = S.tpos[t];
+            if (opening_accept64(pd, tp.x, tp.y, tp.z, T.th2)) am |= 1u << t; else rm |= 1u << t;
             und &= und - 1u;
           } while (und);
         }
