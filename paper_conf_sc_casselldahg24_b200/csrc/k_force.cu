@@ -529,9 +529,13 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   V0Smem<kQuad>& S = s_all[w];
   const float4* qf = kQuad ? in_reg(P.t.qf) : nullptr;
-  const int64_t k0 = P.t_begin + (int64_t(blockIdx.x) * kV0Warps + w) * 32;
+#ifndef NBODY_GROUP
+#define NBODY_GROUP 32
+#endif
+  // design experiment: NBODY_GROUP < 32 targets per warp (lanes >= NBODY_GROUP idle)
+  const int64_t k0 = P.t_begin + (int64_t(blockIdx.x) * kV0Warps + w) * NBODY_GROUP;
   const int64_t k = k0 + lane;
-  const bool active = k < P.t_end;
+  const bool active = k < P.t_end && lane < NBODY_GROUP;
   const uint32_t amask = __ballot_sync(kFull, active);
   if (amask == 0) return;
   const Target T = load_target(P, k, active);
@@ -708,6 +712,8 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       K6STAT(17, __reduce_add_sync(kFull, has && (((m & 0xffffu) == m) || ((m >> 16) << 16) == m)));
       K6STAT(18, __reduce_add_sync(kFull, has ? __popc(m) : 0u));
       K6STAT(24, __reduce_add_sync(kFull, has ? __popc(am) : 0u));
+      K6STAT(29, __reduce_add_sync(kFull, has && g >= leaf0));
+      K6STAT(30, __reduce_add_sync(kFull, has && g >= leaf0 / 2 && g < leaf0));
       K6STAT(25, __reduce_add_sync(kFull, has ? __popc(rm) : 0u));
       if (__any_sync(kFull, und != 0u)) {  // rare: exact fp64 decisions
         if (und) {
@@ -836,7 +842,7 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
     else
       k_force_maskstack<false><<<grid, 32 * kV1Warps, 0, s>>>(p);
   } else {
-    const unsigned grid = unsigned((warps + kV0Warps - 1) / kV0Warps);
+    const unsigned grid = unsigned(((nt + NBODY_GROUP - 1) / NBODY_GROUP + kV0Warps - 1) / kV0Warps);
     const bool soft = p.eps2 > 0.f;
     if (soft && !quad)
       k_force_grouped<true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
