@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle force-sample time")
     ap.add_argument("--exchange", choices=["peer", "nccl"], default="peer",
                     help="multi-GPU exchange: fused update + peer-memory stores (default) or NCCL all-gather")
+    ap.add_argument("--balance", choices=["cost", "equal"], default="cost",
+                    help="multi-GPU ranges (peer exchange): cost-weighted from the last pass (NEXT-3(i), default) "
+                         "or equal slices [A21]")
     ap.add_argument("--sort-every", type=int, default=1,
                     help="ablation: tree reuse, re-sort every k-th step (NEXT-3(iii)); 1 = Alg. 6")
     return ap.parse_args()
@@ -70,6 +73,7 @@ def config_json(cfg, world, extra=None):
     d = {"workload": f"{cfg['workload']} N={cfg['n']} ({args_config_name(cfg)})", "n": cfg["n"],
          "theta": cfg["theta"], "eps": cfg["eps"], "dt": cfg["dt"], "key_bits": 16, "seed": cfg["seed"],
          "sort_every": cfg.get("sort_every", 1), "exchange": cfg.get("exchange", "none"),
+         "balance": cfg.get("balance", "none"),
          "parallelism": "single" if world == 1 else f"hilbert-range x{world}",
          "l2": "inputs larger than L2 (bodies 320 MB + tree ~1 GB per step at N=1e7); no explicit flush"}
     if extra:
@@ -223,6 +227,9 @@ def run_ours(args, cfg, world, rank, local):
     if world > 1:
         if args.exchange == "peer" and world <= 8:
             sim.attach_peers_group(rank, world)
+            if args.balance == "cost":
+                sim.set_option(9, 1)  # NBODY_OPT_BALANCE
+            cfg["balance"] = args.balance
         else:
             sim.attach_process_group(rank, world)
         cfg["exchange"] = sim.exchange_mode()

@@ -89,7 +89,17 @@ enum {
    * (fp64, parallel-axis theorem) and accepted nodes add the softened
    * quadrupole term.  The opening test, hence every interaction list, is
    * unchanged.  Allocates 80 B per internal node on first use. */
-  NBODY_OPT_MULTIPOLE = 8
+  NBODY_OPT_MULTIPOLE = 8,
+  /* NEXT-3(i) cost-weighted Hilbert ranges (P:320 cites
+   * load balance as the scale-out concern): 0 = equal slices [A21]
+   * (default); 1 = after every force pass the ranks re-split the sorted
+   * slots so that each owns about the same number of interactions of that
+   * pass (group costs exchanged over peer memory; boundaries multiples of 32
+   * slots, slices at most 2 ceil(N/32/G) groups), decided on the device and
+   * identical on every rank.  Takes effect only with the fused peer
+   * exchange (nbody_attach_peers*); results stay bit-identical to one GPU.
+   * nbody_get_partition then reports the range of the last force pass. */
+  NBODY_OPT_BALANCE = 9
 };
 
 typedef struct {

@@ -26,6 +26,7 @@ NBODY_OPT_TIMING = 5
 NBODY_OPT_BUILD = 6
 NBODY_OPT_SORT_EVERY = 7
 NBODY_OPT_MULTIPOLE = 8
+NBODY_OPT_BALANCE = 9
 
 _STATUS = {0: "NBODY_OK", -1: "NBODY_EINVAL", -2: "NBODY_ENOMEM", -3: "NBODY_ECUDA", -4: "NBODY_ENCCL",
            -5: "NBODY_ESTATE"}

@@ -92,6 +92,11 @@ struct nbody_ctx {
   unsigned* xflags = nullptr;       // [kBarrierSlots][kMaxPeers] epochs signalled to this rank
   unsigned* xepoch = nullptr;       // [kBarrierSlots] this rank's barrier counters
   int* xerr = nullptr;              // set by a barrier that timed out
+  // NEXT-3(i) cost-weighted ranges (peer exchange only)
+  bool balance = false;
+  uint32_t* gcost = nullptr;        // [ceil(n/32)] interactions per 32-slot group, last pass
+  int64_t* dpart = nullptr;         // [kMaxPeers + 1] slot boundaries of the next pass
+  int64_t* dpart_used = nullptr;    // [kMaxPeers + 1] boundaries of the last pass
 };
 
 namespace {
@@ -213,7 +218,8 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 16 * size_t(inner);                     // bhi
   sz[k++] = 8 * size_t(ids);                        // rc (-inf at the leaves)
   sz[k++] = 16 * size_t(inner);                     // tf
-  sz[k++] = 256;                                    // exchange flags, epochs, error
+  sz[k++] = 4 * size_t(n / 32 + 1);                 // gcost
+  sz[k++] = 512;                                    // exchange flags, epochs, error, partitions
   size_t total = 0;
   for (int i = 0; i < k; ++i) total += align_up(sz[i]);
   cudaError_t e = cudaMalloc(&c->arena, total);
@@ -250,9 +256,12 @@ nbody_status allocate(nbody_ctx* c) {
   c->tree.bhi = (float4*)take();
   c->tree.rc = (float2*)take();
   c->tree.tf = (float4*)take();
+  c->gcost = (uint32_t*)take();
   c->xflags = (unsigned*)take();
   c->xepoch = c->xflags + kBarrierSlots * kMaxPeers;
   c->xerr = reinterpret_cast<int*>(c->xepoch + kBarrierSlots);
+  c->dpart = reinterpret_cast<int64_t*>(reinterpret_cast<char*>(c->xflags) + 128);
+  c->dpart_used = c->dpart + kMaxPeers + 1;
   c->arena_bytes = total;
   c->tree.grid = c->grid;
   c->tree.th2 = c->theta * c->theta;
@@ -261,7 +270,7 @@ nbody_status allocate(nbody_ctx* c) {
   // leaves always interact when reached: thresholds (-inf, -inf), set once
   const float ninf = -INFINITY;
   launch_fill_float2(c->tree.rc + (int64_t(1) << c->tree.L), n, make_float2(ninf, ninf), nullptr);
-  e = cudaMemset(c->xflags, 0, 256);
+  e = cudaMemset(c->xflags, 0, 512);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
   c->sort.n = n;
@@ -269,6 +278,21 @@ nbody_status allocate(nbody_ctx* c) {
   c->sort.ghist = (uint32_t*)sortmem;
   c->sort.tile_ctr = c->sort.ghist + 8 * 256;
   c->sort.status = c->sort.tile_ctr + 8;
+  return NBODY_OK;
+}
+
+// NEXT-3(i) is active: peer exchange over G > 1 ranks with balance on.
+bool balanced(const nbody_ctx* c) { return c->balance && c->xpeer && c->world > 1; }
+
+// Rank q's slot range in the last force pass (host view; syncs when the
+// ranges live on the device).
+nbody_status rank_range(nbody_ctx* c, int q, int64_t* b, int64_t* e) {
+  if (!balanced(c)) return nbody_partition(c->n, q, c->world, b, e);
+  int64_t r[2];
+  CK(cudaStreamSynchronize(c->stream));
+  CK(cudaMemcpy(r, c->dpart_used + q, sizeof(r), cudaMemcpyDeviceToHost));
+  *b = r[0];
+  *e = r[1];
   return NBODY_OK;
 }
 
@@ -347,14 +371,28 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   fp.acc = c->acc;
   fp.count = c->cnt;
   fp.total = c->total;
+  const bool bal = balanced(c);
+  const int64_t groups = (n + 31) / 32;
+  const int64_t cap_groups = std::min(groups, 2 * ((groups + c->world - 1) / c->world));
+  if (bal) {  // NEXT-3(i): the range is read on the device
+    fp.part = c->dpart;
+    fp.part_rank = c->rank;
+    fp.cap = std::min(n, 32 * cap_groups);
+    fp.xp = c->peers;
+  }
   launch_force(fp, c->traversal, s);
   CK(mark(4));
   if (integrate && c->xpeer) {
     // K7 stores the owned records into every rank's state, then the
     // delivery barrier (k_exchange.cu)
-    launch_leapfrog_scatter(c->pm[1], c->vi[1], c->acc, ob, oe - ob, float(c->dt), c->peers, s);
+    launch_leapfrog_scatter(c->pm[1], c->vi[1], c->acc, ob, bal ? fp.cap : oe - ob, float(c->dt), c->peers,
+                            bal ? c->dpart : nullptr, s);
     launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
     ++x_kernels;
+    if (bal) {  // every group cost has landed: next pass's ranges
+      launch_partition(c->gcost, groups, c->world, n, cap_groups, c->dpart, c->dpart_used, s);
+      ++x_kernels;
+    }
   } else if (integrate) {
     launch_leapfrog(c->pm[1] + ob, c->vi[1] + ob, c->acc, oe - ob, float(c->dt), c->pm[0] + ob, c->vi[0] + ob, s);
 #ifdef NBODY_WITH_NCCL
@@ -376,6 +414,10 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     if (c->xpeer) {  // every rank's forces are final before a getter reads them
       launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
       ++x_kernels;
+      if (bal) {
+        launch_partition(c->gcost, groups, c->world, n, cap_groups, c->dpart, c->dpart_used, s);
+        ++x_kernels;
+      }
     }
   }
   CK(mark(5));
@@ -429,11 +471,17 @@ void attach_peer_bases(nbody_ctx* c, char* const* base, int rank, int world) {
     pt.pm[q] = (float4*)at(q, c->pm[0]);
     pt.vi[q] = (float4*)at(q, c->vi[0]);
     pt.flags[q] = (unsigned*)at(q, c->xflags);
+    pt.gcost[q] = (uint32_t*)at(q, c->gcost);
     c->peer_acc[q] = (const float4*)at(q, c->acc);
     c->peer_cnt[q] = (const uint32_t*)at(q, c->cnt);
   }
   set_part(c, rank, world);
   c->xpeer = true;
+  // NEXT-3(i): the first pass uses the equal slices [A21]
+  int64_t bounds[kMaxPeers + 1];
+  for (int q = 0; q <= world; ++q) bounds[q] = std::min(c->n, int64_t(q) * c->own_s);
+  cudaMemcpy(c->dpart, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice);
+  cudaMemcpy(c->dpart_used, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice);
   drop_graph(c);
 }
 
@@ -544,6 +592,11 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "timing must be 0 or 1");
       c->timing = value != 0;
       return NBODY_OK;
+    case NBODY_OPT_BALANCE:
+      if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "balance must be 0 or 1");
+      c->balance = value != 0;
+      drop_graph(c);
+      return NBODY_OK;
     case NBODY_OPT_TRAVERSAL:
       if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown traversal variant");
       c->traversal = int(value);
@@ -640,7 +693,8 @@ nbody_status nbody_sync(nbody_ctx* c) {
 static nbody_status gather_peers(nbody_ctx* c, const void* const* src, void* dst, size_t rec_bytes) {
   for (int q = 0; q < c->world; ++q) {
     int64_t b = 0, e = 0;
-    nbody_partition(c->n, q, c->world, &b, &e);
+    const nbody_status st = rank_range(c, q, &b, &e);
+    if (st != NBODY_OK) return st;
     if (e > b)
       CK(cudaMemcpyAsync(static_cast<char*>(dst) + rec_bytes * size_t(b), src[q], rec_bytes * size_t(e - b),
                          cudaMemcpyDefault, c->stream));
@@ -783,8 +837,13 @@ nbody_status nbody_get_partition(nbody_ctx* c, int* rank, int* world, int64_t* b
   CHECK_CTX(c);
   if (rank) *rank = c->rank;
   if (world) *world = c->world;
-  if (begin) *begin = c->own_b;
-  if (end) *end = c->own_e;
+  int64_t b = c->own_b, e = c->own_e;
+  if (balanced(c)) {  // NEXT-3(i): the range of the last force pass
+    const nbody_status st = rank_range(c, c->rank, &b, &e);
+    if (st != NBODY_OK) return st;
+  }
+  if (begin) *begin = b;
+  if (end) *end = e;
   return NBODY_OK;
 }
 

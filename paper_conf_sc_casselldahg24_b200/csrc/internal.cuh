@@ -54,6 +54,19 @@ struct TreeView {
   float4* qf;      // per internal node, 2 x float4: (Sxx, Syy, Szz, trS), (Sxy, Sxz, Syz, 0)
 };
 
+constexpr int kMaxPeers = 8;                 // one NVSwitch domain of an HGX B200
+constexpr int kBarrierSlots = 2;             // 0: state consumed, 1: state delivered
+// Every rank's state buffers, barrier flags and group costs, mapped into this
+// process (CUDA IPC over NVLink/NVSwitch, or plain pointers for contexts
+// sharing one device).  Index = rank; the own rank's entries are local.
+struct PeerTable {
+  float4* pm[kMaxPeers];
+  float4* vi[kMaxPeers];
+  unsigned* flags[kMaxPeers];                // [kBarrierSlots][kMaxPeers] epochs per rank
+  uint32_t* gcost[kMaxPeers];                // per 32-slot group: interactions of the last pass (NEXT-3(i))
+  int G = 0, rank = 0;
+};
+
 struct ForceParams {
   TreeView t;
   const float4* leaves;   // sorted (x, y, z, m)
@@ -65,6 +78,14 @@ struct ForceParams {
   float4* acc;            // per owned slot (ax, ay, az, 0), indexed slot - t_begin
   uint32_t* count;        // interactions per owned slot
   unsigned long long* total;  // sum of interactions (integer atomics only)
+  // NEXT-3(i) cost-weighted ranges: when part != null the owned range is
+  // [part[part_rank], part[part_rank + 1]) read on the device (t_begin/t_end
+  // ignored; the grid covers cap slots) and every warp stores its group's
+  // interaction count into gcost of every rank in xp.
+  const int64_t* part = nullptr;
+  int part_rank = 0;
+  int64_t cap = 0;
+  PeerTable xp{};
 };
 
 // ---- K1 / K2 --------------------------------------------------------------
@@ -123,21 +144,17 @@ void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s);
 
 // ---- K7 fused with the exchange over peer memory -------------
-// Every rank's state buffers and barrier flags, mapped into this process
-// (CUDA IPC over NVLink/NVSwitch, or plain pointers for contexts sharing one
-// device).  Index = rank; the own rank's entries are local pointers.
-constexpr int kMaxPeers = 8;                 // one NVSwitch domain of an HGX B200
-constexpr int kBarrierSlots = 2;             // 0: state consumed, 1: state delivered
-struct PeerTable {
-  float4* pm[kMaxPeers];
-  float4* vi[kMaxPeers];
-  unsigned* flags[kMaxPeers];                // [kBarrierSlots][kMaxPeers] epochs per rank
-  int G = 0, rank = 0;
-};
 // Leapfrog of the owned slots [b, b + len) (acc indexed from 0), storing the
 // new records straight into slot b + i of EVERY rank's pm0/vi0.
+// With part != null the range is [part[rank], part[rank + 1]) read on the
+// device and len is only the launch bound (cap).
 void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t b, int64_t len,
-                             float dt, const PeerTable& pt, cudaStream_t s);
+                             float dt, const PeerTable& pt, const int64_t* part, cudaStream_t s);
+// NEXT-3(i): next step's cost-weighted ranges from the group costs of the
+// last pass (identical on every rank): part[0..G] <- boundaries (multiples of
+// 32 slots, each slice <= cap_groups groups); used[0..G] <- the old part.
+void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_groups, int64_t* part,
+                      int64_t* used, cudaStream_t s);
 // Device-side barrier over the G ranks: signal epoch+1 of `slot` to every
 // rank (release, system scope), then wait until every rank's signal for
 // that epoch arrived in the own flag block (acquire).  A wait longer than

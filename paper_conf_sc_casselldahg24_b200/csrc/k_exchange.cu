@@ -38,7 +38,11 @@ __device__ __forceinline__ uint64_t global_ns() {
 __global__ __launch_bounds__(256) void k_leapfrog_scatter(const float4* __restrict__ pm_in,
                                                           const float4* __restrict__ vi_in,
                                                           const float4* __restrict__ acc, int64_t b, int64_t len,
-                                                          float dt, PeerTable pt) {
+                                                          float dt, PeerTable pt, const int64_t* __restrict__ part) {
+  if (part) {  // NEXT-3(i): this step's range, decided on the device
+    b = part[pt.rank];
+    len = part[pt.rank + 1] - b;
+  }
   const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (i >= len) return;
   float4 p = pm_in[b + i], v = vi_in[b + i];
@@ -55,6 +59,67 @@ __global__ __launch_bounds__(256) void k_leapfrog_scatter(const float4* __restri
     if (r < pt.G) {
       pt.pm[r][b + i] = p;
       pt.vi[r][b + i] = v;
+    }
+  }
+}
+
+// NEXT-3(i) cost-weighted Hilbert ranges.  Group j (32
+// slots) costs w_j = its interaction count in the last pass (identical data
+// on every rank after the delivery barrier).  With E_j = sum_{i<j} w_i and
+// W = E_J, boundary r is B_r = min{ j : E_j >= ceil(r W / G) }, then clamped
+// in rank order so that every slice has at most cap_groups groups and the
+// remaining ranks can still cover the rest; slot boundary = min(n, 32 B_r).
+// One block: each thread sums a contiguous chunk, a block scan of the chunk
+// sums locates the chunk holding each target, whose thread walks it.
+constexpr int kPartThreads = 1024;
+
+__global__ __launch_bounds__(kPartThreads) void k_partition(const uint32_t* __restrict__ w, int64_t J, int G,
+                                                            int64_t n, int64_t cap, int64_t* __restrict__ part,
+                                                            int64_t* __restrict__ used) {
+  __shared__ unsigned long long s_pre[kPartThreads + 1];
+  __shared__ int64_t s_B[kMaxPeers + 1];
+  const int t = threadIdx.x;
+  const int64_t chunk = (J + kPartThreads - 1) / kPartThreads;
+  const int64_t j0 = min(J, int64_t(t) * chunk), j1 = min(J, j0 + chunk);
+  unsigned long long sum = 0;
+  for (int64_t j = j0; j < j1; ++j) sum += w[j];
+  s_pre[t + 1] = sum;
+  if (t == 0) s_pre[0] = 0;
+  __syncthreads();
+  for (int o = 1; o < kPartThreads; o <<= 1) {  // inclusive scan of s_pre[1..]
+    const unsigned long long v = t >= o ? s_pre[t + 1 - o] : 0ull;
+    __syncthreads();
+    s_pre[t + 1] += v;
+    __syncthreads();
+  }
+  const unsigned long long W = s_pre[kPartThreads];
+  // thread t owns targets with s_pre[t] < target <= s_pre[t + 1]
+  for (int r = 1; r < G; ++r) {
+    using u64 = unsigned long long;
+    const u64 target = (W * u64(r) + u64(G) - 1) / u64(G);
+    if (target == 0) {
+      if (t == 0) s_B[r] = 0;
+    } else if (s_pre[t] < target && target <= s_pre[t + 1]) {
+      unsigned long long e = s_pre[t];
+      int64_t j = j0;
+      while (e < target) e += w[j++];  // E_j >= target first at this j
+      s_B[r] = j;
+    }
+  }
+  __syncthreads();
+  if (t == 0) {
+    s_B[0] = 0;
+    s_B[G] = J;
+    for (int r = 1; r < G; ++r) {
+      int64_t b = s_B[r];
+      b = max(b, s_B[r - 1]);
+      b = min(b, s_B[r - 1] + cap);
+      b = max(b, J - int64_t(G - r) * cap);
+      s_B[r] = b;
+    }
+    for (int r = 0; r <= G; ++r) {
+      used[r] = part[r];
+      part[r] = min(n, 32 * s_B[r]);
     }
   }
 }
@@ -87,9 +152,14 @@ __global__ void k_xbarrier(PeerTable pt, unsigned* epoch, int slot, int* err) {
 }  // namespace
 
 void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t b, int64_t len,
-                             float dt, const PeerTable& pt, cudaStream_t s) {
+                             float dt, const PeerTable& pt, const int64_t* part, cudaStream_t s) {
   if (len <= 0) return;
-  k_leapfrog_scatter<<<unsigned((len + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, b, len, dt, pt);
+  k_leapfrog_scatter<<<unsigned((len + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, b, len, dt, pt, part);
+}
+
+void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_groups, int64_t* part,
+                      int64_t* used, cudaStream_t s) {
+  k_partition<<<1, kPartThreads, 0, s>>>(gcost, groups, G, n, cap_groups, part, used);
 }
 
 void launch_xbarrier(const PeerTable& pt, unsigned* epoch, int slot, int* err, cudaStream_t s) {

@@ -291,13 +291,30 @@ __device__ __forceinline__ Target load_target(const ForceParams& P, int64_t k, b
   return T;
 }
 
-__device__ __forceinline__ void store_result(const ForceParams& P, int64_t k, bool active, const Acc& a, int lane) {
+// The owned target range: static, or (NEXT-3(i)) read from the device.
+__device__ __forceinline__ void owned_range(const ForceParams& P, int64_t& tb, int64_t& te) {
+  if (P.part) {
+    tb = P.part[P.part_rank];
+    te = P.part[P.part_rank + 1];
+  } else {
+    tb = P.t_begin;
+    te = P.t_end;
+  }
+}
+
+// k: this lane's slot; k0: the warp's first slot (a multiple of 32 from 0).
+__device__ __forceinline__ void store_result(const ForceParams& P, int64_t tb, int64_t k, int64_t k0, bool active,
+                                             const Acc& a, int lane) {
   if (active) {
-    P.acc[k - P.t_begin] = make_float4(a.x, a.y, a.z, 0.f);
-    P.count[k - P.t_begin] = a.n;
+    P.acc[k - tb] = make_float4(a.x, a.y, a.z, 0.f);
+    P.count[k - tb] = a.n;
   }
   const uint32_t tot = __reduce_add_sync(kFull, active ? a.n : 0u);
-  if (lane == 0) atomicAdd(P.total, (unsigned long long)tot);
+  if (lane == 0) {
+    atomicAdd(P.total, (unsigned long long)tot);
+    if (P.part)  // NEXT-3(i): this group's cost, to every rank
+      for (int q = 0; q < P.xp.G; ++q) P.xp.gcost[q][k0 >> 5] = tot;
+  }
 }
 
 // ------------------------------------------------------------ variant 1 ----
@@ -306,8 +323,11 @@ constexpr int kV1Warps = 8;
 template <bool kQuad>
 __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForceParams P) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t k = P.t_begin + (int64_t(blockIdx.x) * kV1Warps + w) * 32 + lane;
-  const bool active = k < P.t_end;
+  int64_t tb, te;
+  owned_range(P, tb, te);
+  const int64_t k0 = tb + (int64_t(blockIdx.x) * kV1Warps + w) * 32;
+  const int64_t k = k0 + lane;
+  const bool active = k < te;
   const uint32_t amask = __ballot_sync(kFull, active);
   if (amask == 0) return;
   const Target T = load_target(P, k, active);
@@ -315,7 +335,7 @@ __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForcePa
   const Walk W = make_walk(P);
   const uint32_t kid = W.leaf0 + uint32_t(k);
   mask_walk<kQuad>(W, T, kid, a, lane, 1u, amask);
-  store_result(P, k, active, a, lane);
+  store_result(P, tb, k, k0, active, a, lane);
 }
 
 
@@ -533,9 +553,11 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
 #define NBODY_GROUP 32
 #endif
   // design experiment: NBODY_GROUP < 32 targets per warp (lanes >= NBODY_GROUP idle)
-  const int64_t k0 = P.t_begin + (int64_t(blockIdx.x) * kV0Warps + w) * NBODY_GROUP;
+  int64_t tb, te;
+  owned_range(P, tb, te);
+  const int64_t k0 = tb + (int64_t(blockIdx.x) * kV0Warps + w) * NBODY_GROUP;
   const int64_t k = k0 + lane;
-  const bool active = k < P.t_end && lane < NBODY_GROUP;
+  const bool active = k < te && lane < NBODY_GROUP;
   const uint32_t amask = __ballot_sync(kFull, active);
   if (amask == 0) return;
   const Target T = load_target(P, k, active);
@@ -821,7 +843,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
     }
   }
   flush(true);
-  store_result(P, k, active, a, lane);
+  store_result(P, tb, k, k0, active, a, lane);
 #ifdef NBODY_K6_STATS
   if (lane == 0)
     for (int i = 0; i < kK6Stats; ++i) atomicAdd(&g_k6_stats[i], st[i]);
@@ -831,7 +853,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
 }  // namespace
 
 void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
-  const int64_t nt = p.t_end - p.t_begin;
+  const int64_t nt = p.part ? p.cap : p.t_end - p.t_begin;
   if (nt <= 0) return;
   const int64_t warps = (nt + 31) / 32;
   const bool quad = p.t.quad;

@@ -46,7 +46,8 @@ class NBody:
     """One simulation context: ``NBody(n, theta, eps, dt)``."""
 
     def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
-                 stream=None, use_graph: bool = True, traversal: int = 0, device=None, multipole: int = 1):
+                 stream=None, use_graph: bool = True, traversal: int = 0, device=None, multipole: int = 1,
+                 balance: bool = False):
         self.lib = _capi.load()
         self.n = int(n)
         if device is None:  # follow PyTorch's current device when torch has one
@@ -70,6 +71,8 @@ class NBody:
         self.set_option(_capi.NBODY_OPT_TRAVERSAL, traversal)
         if multipole != 1:
             self.set_option(_capi.NBODY_OPT_MULTIPOLE, multipole)
+        if balance:  # NEXT-3(i) cost-weighted ranges (peer exchange only)
+            self.set_option(_capi.NBODY_OPT_BALANCE, 1)
         if stream is not None:
             self.set_option(_capi.NBODY_OPT_STREAM, int(stream))
 

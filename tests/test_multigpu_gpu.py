@@ -105,6 +105,10 @@ def _run_peer_local(NB, pos, vel, mass, world, steps, **kw):
     (4, 30_001, {"use_graph": False}),
     (2, 25_000, {"multipole": 2}),
     (3, 12_345, {"traversal": 1}),
+    (2, 20_000, {"balance": True}),
+    (8, 40_000, {"balance": True}),
+    (4, 30_001, {"balance": True, "use_graph": False}),
+    (3, 12_345, {"balance": True, "traversal": 1}),
 ])
 def test_peer_exchange_is_bit_identical(NB, world, n, kw):
     """G contexts on one GPU exchange through k_leapfrog_scatter's stores into
@@ -126,6 +130,78 @@ def test_peer_exchange_is_bit_identical(NB, world, n, kw):
         assert (s.get_interactions() == c_ref).all()
         total += s.stats()["interactions"]
     assert total == ref.stats()["interactions"]
+
+
+def _expected_bounds(counts_by_slot, world):
+    """NEXT-3(i) rule (k_exchange.cu k_partition), restated in numpy: group j
+    (32 slots) costs the sum of its slots' interaction counts; boundary r is
+    the first j with E_j = sum_{i<j} w_i >= ceil(r W / G), clamped so that no
+    slice exceeds 2 ceil(J / G) groups; slot boundary min(n, 32 B_r)."""
+    n = len(counts_by_slot)
+    J = (n + 31) // 32
+    w = np.zeros(J * 32, np.int64)
+    w[:n] = counts_by_slot
+    w = w.reshape(J, 32).sum(1)
+    E = np.concatenate([[0], np.cumsum(w)])
+    W = int(E[-1])
+    cap = min(J, 2 * ((J + world - 1) // world))
+    B = [0]
+    for r in range(1, world):
+        t = -(-W * r // world)
+        b = int(np.searchsorted(E, t, side="left")) if t > 0 else 0
+        b = max(b, B[-1])
+        b = min(b, B[-1] + cap)
+        b = max(b, J - (world - r) * cap)
+        B.append(b)
+    B.append(J)
+    return [min(n, 32 * b) for b in B]
+
+
+@pytest.mark.parametrize("world,workload", [(2, "clustered"), (4, "disks"), (8, "clustered")])
+def test_balanced_ranges_follow_last_pass_costs(NB, world, workload):
+    """NEXT-3(i): after a step, the ranges of the next force pass are the
+    cost-weighted split of the previous pass's per-slot interaction counts,
+    identical on every rank; results stay bit-identical to one GPU and the
+    per-rank interaction counts are balanced at least as well as equal
+    slices."""
+    n = 50_000
+    pos, vel, mass = generate(workload, n, 70 + world)
+    ref = NB(n, 0.5, 1e-3, 1e-3)
+    ref.set_bodies(pos, vel, mass)
+    ranks = [NB(n, 0.5, 1e-3, 1e-3, balance=True) for _ in range(world)]
+    NB.attach_peers_local(ranks)
+    for s in ranks:
+        s.set_bodies(pos, vel, mass)
+    eq = [s.partition()[2:] for s in ranks]
+    prev_counts = None
+    for step in range(4):
+        ref.step(1)
+        for s in ranks:
+            s.step(1)
+        for s in ranks:
+            s.sync()
+        got = [s.partition()[2:] for s in ranks]
+        assert all(got[r][1] == got[r + 1][0] for r in range(world - 1))
+        assert got[0][0] == 0 and got[-1][1] == n
+        assert all(b % 32 == 0 for b, _ in got)
+        if prev_counts is None:
+            assert got == eq                      # the first pass uses the equal slices
+        else:
+            exp = _expected_bounds(prev_counts, world)
+            assert [b for b, _ in got] == exp[:-1] and got[-1][1] == exp[-1]
+        _, vi = ref.get_state()                   # slot order of this pass
+        ids = vi[:, 3].view(np.uint32)
+        prev_counts = ref.get_interactions()[ids].astype(np.int64)
+        for s in ranks:
+            assert (s.get_positions() == ref.get_positions()).all()
+            assert (s.get_interactions() == ref.get_interactions()).all()
+    # balance of the last pass: per-rank interactions vs equal slices
+    per_rank = [s.stats()["interactions"] for s in ranks]
+    assert sum(per_rank) == ref.stats()["interactions"]
+    _, vi = ref.get_state()
+    cnt = ref.get_interactions()[vi[:, 3].view(np.uint32)].astype(np.int64)
+    eq_cost = [int(cnt[b:e].sum()) for b, e in eq]
+    assert max(per_rank) / np.mean(per_rank) <= max(eq_cost) / np.mean(eq_cost) + 1e-9
 
 
 def test_peer_exchange_tree_reuse_and_compute_accel(NB):
