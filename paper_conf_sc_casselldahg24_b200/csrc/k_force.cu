@@ -735,6 +735,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       K6STAT(18, __reduce_add_sync(kFull, has ? __popc(m) : 0u));
       K6STAT(24, __reduce_add_sync(kFull, has ? __popc(am) : 0u));
       K6STAT(29, __reduce_add_sync(kFull, has && g >= leaf0));
+      K6STAT(31, __reduce_add_sync(kFull, has && g < leaf0 && (am == m || (rm == m))));
       K6STAT(30, __reduce_add_sync(kFull, has && g >= leaf0 / 2 && g < leaf0));
       K6STAT(25, __reduce_add_sync(kFull, has ? __popc(rm) : 0u));
       if (__any_sync(kFull, und != 0u)) {  // rare: exact fp64 decisions

@@ -18,7 +18,7 @@ kStatNames = ["warps", "A batches", "A nodes", "T batches", "T nodes", "full ent
               "dense_part calls", "dense_part pairs", "spill walks", "T batches < 32",
               "T nodes 1-quarter", "T nodes 1-half", "T mask lanes", "partial q-incid", "partial 1-quarter",
               "partial h-incid", "part sum max q", "part sum max h", "T accept lanes", "T open lanes",
-              "part max 8grp", "part max 16grp", "part max lane", "T leaf nodes", "T level-1 nodes", "-"]
+              "part max 8grp", "part max 16grp", "part max lane", "T leaf nodes", "T level-1 nodes", "T internal uniform"]
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="disks")
