@@ -7,6 +7,11 @@ reading in DESIGN.md.
 
 ``step()`` composes Alg. 6 from the C++ pieces:
 bbox -> keys -> stable sort -> permute -> build -> force -> leapfrog (O8).
+
+``precision=32`` (default): fp32 bodies, the state precision of the path
+under test.  ``precision=64`` (NEXT-2): fp64 bodies and state -- the paper's
+own precision throughout; every stage evaluates the same
+expressions on the doubles.
 """
 from __future__ import annotations
 
@@ -69,8 +74,16 @@ def lib():
         L.orc_force_list.argtypes = [_P, C.c_double, C.c_double, C.c_int64, _i64p, C.c_int64]
         L.orc_force_list.restype = C.c_int64
         L.orc_direct.argtypes = [C.c_int64, _f32p, _f32p, C.c_double, _i64p, C.c_int64, _f64p, C.c_int]
+        L.orc_bbox_d.argtypes = [C.c_int64, _f64p, _f64p, _f64p]
+        L.orc_quantize_d.argtypes = [C.c_int64, _f64p, _f64p, _f64p, C.c_int, _u32p]
+        L.orc_keys_d.argtypes = [C.c_int64, _f64p, C.c_int, _u64p]
+        L.orc_build_d.argtypes = [C.c_int64, _f64p, _f64p]
+        L.orc_build_d.restype = _P
+        L.orc_tree_level_box_d.argtypes = [_P, C.c_int, _f64p, _f64p]
+        L.orc_direct_d.argtypes = [C.c_int64, _f64p, _f64p, C.c_double, _i64p, C.c_int64, _f64p, C.c_int]
         for f in ("orc_bbox", "orc_quantize", "orc_keys", "orc_sort", "orc_tree_levels", "orc_tree_level",
-                  "orc_force", "orc_direct"):
+                  "orc_force", "orc_direct", "orc_bbox_d", "orc_quantize_d", "orc_keys_d", "orc_tree_level_box_d",
+                  "orc_direct_d"):
             getattr(L, f).restype = C.c_int
         _lib = L
     return _lib
@@ -83,6 +96,16 @@ def _ok(rc: int, what: str):
 
 def _f32(a, shape=None):
     a = np.ascontiguousarray(a, np.float32)
+    if shape is not None:
+        a = a.reshape(shape)
+    return a
+
+
+def _real(a, precision, shape=None):
+    """fp32 or fp64 contiguous array for the given precision (32 or 64)."""
+    if precision not in (32, 64):
+        raise ValueError("precision must be 32 or 64")
+    a = np.ascontiguousarray(a, np.float32 if precision == 32 else np.float64)
     if shape is not None:
         a = a.reshape(shape)
     return a
@@ -103,29 +126,32 @@ def hilbert_index(x: int, y: int, z: int, b: int) -> int:
     return int(lib().orc_hilbert_index(x, y, z, b))
 
 
-def bbox(pos):
+def bbox(pos, precision: int = 32):
     """O1 -- Alg. 3 (P:79-97)."""
-    pos = _f32(pos, (-1, 3))
-    lo = np.empty(3, np.float32)
-    hi = np.empty(3, np.float32)
-    _ok(lib().orc_bbox(len(pos), pos, lo, hi), "bbox")
+    pos = _real(pos, precision, (-1, 3))
+    lo = np.empty(3, pos.dtype)
+    hi = np.empty(3, pos.dtype)
+    f = lib().orc_bbox if precision == 32 else lib().orc_bbox_d
+    _ok(f(len(pos), pos, lo, hi), "bbox")
     return lo, hi
 
 
-def quantize(pos, b: int):
+def quantize(pos, b: int, precision: int = 32):
     """O2 -- grid cells [A9][A17]."""
-    pos = _f32(pos, (-1, 3))
-    lo, hi = bbox(pos)
+    pos = _real(pos, precision, (-1, 3))
+    lo, hi = bbox(pos, precision)
     q = np.empty((len(pos), 3), np.uint32)
-    _ok(lib().orc_quantize(len(pos), pos, lo, hi, int(b), q), "quantize")
+    f = lib().orc_quantize if precision == 32 else lib().orc_quantize_d
+    _ok(f(len(pos), pos, lo, hi, int(b), q), "quantize")
     return q
 
 
-def keys(pos, b: int):
+def keys(pos, b: int, precision: int = 32):
     """O1..O3 -- Hilbert key per body in current slot order."""
-    pos = _f32(pos, (-1, 3))
+    pos = _real(pos, precision, (-1, 3))
     out = np.empty(len(pos), np.uint64)
-    _ok(lib().orc_keys(len(pos), pos, int(b), out), "keys")
+    f = lib().orc_keys if precision == 32 else lib().orc_keys_d
+    _ok(f(len(pos), pos, int(b), out), "keys")
     return out
 
 
@@ -143,8 +169,8 @@ class LevelData:
     M: np.ndarray      # fp64 [c]
     com: np.ndarray    # fp64 [c,3]
     s2: np.ndarray     # fp64 [c]
-    lo: np.ndarray     # fp32 [c,3]
-    hi: np.ndarray     # fp32 [c,3]
+    lo: np.ndarray     # fp32 [c,3] (fp64 for a precision-64 tree)
+    hi: np.ndarray     # fp32 [c,3] (fp64 for a precision-64 tree)
 
     @property
     def m32(self):
@@ -158,13 +184,15 @@ class LevelData:
 class Tree:
     """O6 -- BUILDTREEACCUMULATEMASS over Hilbert-sorted bodies."""
 
-    def __init__(self, pos_sorted, mass_sorted):
-        self.pos = _f32(pos_sorted, (-1, 3))
-        self.mass = _f32(mass_sorted, (-1,))
+    def __init__(self, pos_sorted, mass_sorted, precision: int = 32):
+        self.precision = precision
+        self.pos = _real(pos_sorted, precision, (-1, 3))
+        self.mass = _real(mass_sorted, precision, (-1,))
         if len(self.pos) != len(self.mass) or len(self.pos) < 1:
             raise ValueError("bad tree input")
         self.n = len(self.pos)
-        self._h = lib().orc_build(self.n, self.pos, self.mass)
+        build_fn = lib().orc_build if precision == 32 else lib().orc_build_d
+        self._h = build_fn(self.n, self.pos, self.mass)
         if not self._h:
             raise MemoryError("orc_build failed")
         self.L = lib().orc_tree_levels(self._h)
@@ -186,6 +214,10 @@ class Tree:
                       np.empty((c, 3), np.float32))
         _ok(lib().orc_tree_level(self._h, l, d.M.ctypes.data, d.com.ctypes.data, d.s2.ctypes.data,
                                  d.lo.ctypes.data, d.hi.ctypes.data), "tree_level")
+        if self.precision == 64:
+            d.lo = np.empty((c, 3))
+            d.hi = np.empty((c, 3))
+            _ok(lib().orc_tree_level_box_d(self._h, l, d.lo, d.hi), "tree_level_box_d")
         return d
 
     def force(self, theta: float, eps: float, targets=None, nthreads: int = 0, quad: bool = False):
@@ -214,13 +246,15 @@ class Tree:
         return out[: 2 * c].reshape(c, 2)
 
 
-def direct(pos, mass, eps: float, targets=None, nthreads: int = 0):
-    """D -- direct summation of Eq. 1, softened, fp64."""
-    pos = _f32(pos, (-1, 3))
-    mass = _f32(mass, (-1,))
+def direct(pos, mass, eps: float, targets=None, nthreads: int = 0, precision: int = 32):
+    """D -- direct summation of Eq. 1, softened, fp64 arithmetic on
+    fp32 (precision=32) or fp64 (precision=64) bodies."""
+    pos = _real(pos, precision, (-1, 3))
+    mass = _real(mass, precision, (-1,))
     t = np.arange(len(pos), dtype=np.int64) if targets is None else np.ascontiguousarray(targets, np.int64)
     acc = np.empty((len(t), 3))
-    _ok(lib().orc_direct(len(pos), pos, mass, float(eps), t, len(t), acc, int(nthreads)), "direct")
+    f = lib().orc_direct if precision == 32 else lib().orc_direct_d
+    _ok(f(len(pos), pos, mass, float(eps), t, len(t), acc, int(nthreads)), "direct")
     return acc
 
 
@@ -233,20 +267,22 @@ class StepResult:
     acc: np.ndarray         # fp64 [nt,3] for `targets` (sorted slots)
     count: np.ndarray       # int64 [nt]
     targets: np.ndarray     # sorted slots the force was evaluated for
-    pos: np.ndarray         # fp32 [n,3] sorted, after the update (if integrated)
-    vel: np.ndarray         # fp32 [n,3] sorted, after the update
-    mass: np.ndarray        # fp32 [n] sorted
+    pos: np.ndarray         # fp32 [n,3] sorted, after the update (if integrated); fp64 at precision 64
+    vel: np.ndarray         # fp32 [n,3] sorted, after the update; fp64 at precision 64
+    mass: np.ndarray        # fp32 [n] sorted; fp64 at precision 64
     ids: np.ndarray         # int64 [n]: body id in each sorted slot
     seconds: float
 
 
 def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_bits: int = 16,
          integrate: bool = True, targets=None, nthreads: int = 0, resort: bool = True,
-         quad: bool = False) -> StepResult:
+         quad: bool = False, precision: int = 32) -> StepResult:
     """One step of Alg. 6 on fp32 state in the current slot order.
 
     O8 [A14] kick-drift leapfrog, v_{+1/2} = v_{-1/2} + a dt, x += v_{+1/2} dt,
     evaluated in fp64 and stored in fp32 (the state precision of the path).
+    ``precision=64`` (NEXT-2): fp64 state in, fp64 state out, every stage on
+    the doubles (the paper's precision).
     With ``targets`` (sorted slots) only those bodies get forces and the
     update is skipped.
 
@@ -256,26 +292,26 @@ def step(pos, vel, mass, ids=None, *, theta: float, eps: float, dt: float, key_b
     rebuilt bottom-up over that order at the current positions.
     """
     t0 = time.perf_counter()
-    pos = _f32(pos, (-1, 3))
-    vel = _f32(vel, (-1, 3))
-    mass = _f32(mass, (-1,))
+    pos = _real(pos, precision, (-1, 3))
+    vel = _real(vel, precision, (-1, 3))
+    mass = _real(mass, precision, (-1,))
     n = len(pos)
     ids = np.arange(n, dtype=np.int64) if ids is None else np.asarray(ids, np.int64)
     if resort:
         b = resolve_key_bits(n, key_bits)
-        k = keys(pos, b)                       # O1-O3
+        k = keys(pos, b, precision)            # O1-O3
         perm = sort_perm(k)                    # O4
     else:
         k = np.zeros(0, np.uint64)
         perm = np.arange(n, dtype=np.uint32)
     ps, vs, ms, ids_s = pos[perm], vel[perm], mass[perm], ids[perm]  # O5 [A11]
-    tree = Tree(ps, ms)                        # O6
+    tree = Tree(ps, ms, precision)             # O6
     full = targets is None
     tg = np.arange(n, dtype=np.int64) if full else np.ascontiguousarray(targets, np.int64)
     acc, cnt = tree.force(theta, eps, tg, nthreads, quad)   # O7 (+ NEXT-4 quadrupoles)
     if integrate and full:                     # O8
         v_new = vs.astype(np.float64) + acc * dt
         x_new = ps.astype(np.float64) + v_new * dt
-        vs = v_new.astype(np.float32)
-        ps = x_new.astype(np.float32)
+        vs = v_new.astype(pos.dtype)
+        ps = x_new.astype(pos.dtype)
     return StepResult(k, perm, tree, acc, cnt, tg, ps, vs, ms, ids_s, time.perf_counter() - t0)

@@ -133,25 +133,30 @@ _CHUNKERS = {
 }
 
 
-def generate(name: str, n: int, seed: int):
+def generate(name: str, n: int, seed: int, dtype=np.float32):
     """Return (pos float32[n,3], vel float32[n,3], mass float32[n]).
 
     ``vel`` is read as v_{-1/2} by the leapfrog (reading A14).
+    ``dtype=np.float64`` returns the same fp64 draws without the final cast
+    (inputs of the FP64 mode, NEXT-2); mass is then 1/N in fp64.
     """
+    dtype = np.dtype(dtype)
+    if dtype not in (np.float32, np.float64):
+        raise ValueError("dtype must be float32 or float64")
     if name not in _CHUNKERS:
         raise ValueError(f"unknown workload {name!r}; expected one of {NAMES}")
     n = int(n)
     if n < 1:
         raise ValueError("n must be >= 1")
-    pos = np.empty((n, 3), np.float32)
-    vel = np.empty((n, 3), np.float32)
+    pos = np.empty((n, 3), dtype)
+    vel = np.empty((n, 3), dtype)
     f = _CHUNKERS[name]
     for c, lo in enumerate(range(0, n, CHUNK)):
         hi = min(n, lo + CHUNK)
         p, v = f(_rng(seed, c), lo, hi, n, seed)
         pos[lo:hi] = p
         vel[lo:hi] = v
-    mass = np.full(n, np.float32(1.0 / n), np.float32)
+    mass = np.full(n, dtype.type(1.0 / n), dtype)
     return pos, vel, mass
 
 
