@@ -99,7 +99,18 @@ enum {
    * identical on every rank.  Takes effect only with the fused peer
    * exchange (nbody_attach_peers*); results stay bit-identical to one GPU.
    * nbody_get_partition then reports the range of the last force pass. */
-  NBODY_OPT_BALANCE = 9
+  NBODY_OPT_BALANCE = 9,
+  /* NEXT-2 FP64 mode (the paper's own precision: "FP64" throughout, P:272,
+   * footnote P:282): 32 (default) or 64.  In mode 64 the state (positions,
+   * velocities, masses), the bounding box, the key quantisation, the tree
+   * boxes and moments, every interaction and the leapfrog are fp64; the
+   * opening decisions are the same fp64 test as in mode 32 (fp32 filters
+   * with rigorous bounds decide the clear cases).  Load bodies with
+   * nbody_set_bodies64 and read them with the *64 getters (the fp32 getters
+   * round).  Setting the option drops the loaded bodies.  Mode 64 needs a
+   * single rank (no exchange), monopole order and traversal variant 0
+   * (NBODY_EINVAL otherwise); it allocates about 3.7 GB at N = 10^7. */
+  NBODY_OPT_PRECISION = 10
 };
 
 typedef struct {
@@ -140,6 +151,10 @@ nbody_status nbody_set_option(nbody_ctx *ctx, int option, int64_t value);
  * ids to array indices.  Masses must be > 0 and finite, positions and
  * velocities finite [A18]. */
 nbody_status nbody_set_bodies(nbody_ctx *ctx, const float *pos, const float *vel, const float *mass);
+/* NEXT-2 FP64 mode (NBODY_OPT_PRECISION = 64): as nbody_set_bodies with
+ * fp64 pos[n][3], vel[n][3], mass[n] (host or device; copied).
+ * NBODY_EINVAL in mode 32, for null pointers or invalid values [A18]. */
+nbody_status nbody_set_bodies64(nbody_ctx *ctx, const double *pos, const double *vel, const double *mass);
 
 /* Stages 1-5 of Alg. 6 at the current positions (no UPDATEPOSITION):
  * bbox, keys, sort, permute, build, force.  Afterwards slot order is the
@@ -159,6 +174,11 @@ nbody_status nbody_get_accel(nbody_ctx *ctx, float *out);
 /* Current positions / velocities, out[n][3] by id (fp32). */
 nbody_status nbody_get_positions(nbody_ctx *ctx, float *out);
 nbody_status nbody_get_velocities(nbody_ctx *ctx, float *out);
+/* NEXT-2 FP64 mode: the same outputs in fp64 ([n][3], by body id; host or
+ * device out).  NBODY_EINVAL in mode 32. */
+nbody_status nbody_get_accel64(nbody_ctx *ctx, double *out);
+nbody_status nbody_get_positions64(nbody_ctx *ctx, double *out);
+nbody_status nbody_get_velocities64(nbody_ctx *ctx, double *out);
 
 /* Interactions per body of the last force pass, out[n] by id. */
 nbody_status nbody_get_interactions(nbody_ctx *ctx, uint32_t *out);
@@ -166,6 +186,10 @@ nbody_status nbody_get_interactions(nbody_ctx *ctx, uint32_t *out);
 /* Full state in slot order: pos_m[n][4] = (x, y, z, m), vel_id[n][4] =
  * (vx, vy, vz, id reinterpreted as float bits). */
 nbody_status nbody_get_state(nbody_ctx *ctx, float *pos_m, float *vel_id);
+/* NEXT-2 FP64 mode: the state in slot order, pos_m[n][4] = (x, y, z, m),
+ * vel_id[n][4] = (vx, vy, vz, id as an exact integer); either may be NULL.
+ * NBODY_EINVAL in mode 32 (and nbody_get_state is NBODY_EINVAL in mode 64). */
+nbody_status nbody_get_state64(nbody_ctx *ctx, double *pos_m, double *vel_id);
 
 nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
 
@@ -252,6 +276,11 @@ nbody_status nbody_debug_perm(nbody_ctx *ctx, uint32_t *perm);
  * interaction); box[count][6] fp32 = (lo xyz, hi xyz).  Any of pred, rec,
  * box may be NULL; pass all NULL to query *count. */
 nbody_status nbody_debug_level(nbody_ctx *ctx, int level, int64_t *count, double *pred, float *rec, float *box);
+/* NEXT-2 FP64 mode, after nbody_compute_accel: level l in [1, L]:
+ * rec64[count][4] = (com64, M) and box64[count][6] = (lo xyz, hi xyz) in
+ * fp64; either may be NULL.  (nbody_debug_level's fp32 box is NBODY_EINVAL
+ * in mode 64.) */
+nbody_status nbody_debug_level64(nbody_ctx *ctx, int level, int64_t *count, double *rec64, double *box64);
 
 /* NEXT-4: second mass moments about the COM of level l in [1, L] after
  * nbody_compute_accel with NBODY_OPT_MULTIPOLE = 2: S[count][6] fp64 =

@@ -27,6 +27,7 @@ NBODY_OPT_BUILD = 6
 NBODY_OPT_SORT_EVERY = 7
 NBODY_OPT_MULTIPOLE = 8
 NBODY_OPT_BALANCE = 9
+NBODY_OPT_PRECISION = 10
 
 _STATUS = {0: "NBODY_OK", -1: "NBODY_EINVAL", -2: "NBODY_ENOMEM", -3: "NBODY_ECUDA", -4: "NBODY_ENCCL",
            -5: "NBODY_ESTATE"}
@@ -65,6 +66,12 @@ SIGNATURES = {
     "nbody_get_velocities": (_S, [_P, _P]),
     "nbody_get_interactions": (_S, [_P, _P]),
     "nbody_get_state": (_S, [_P, _P, _P]),
+    "nbody_set_bodies64": (_S, [_P, _P, _P, _P]),
+    "nbody_get_accel64": (_S, [_P, _P]),
+    "nbody_get_positions64": (_S, [_P, _P]),
+    "nbody_get_velocities64": (_S, [_P, _P]),
+    "nbody_get_state64": (_S, [_P, _P, _P]),
+    "nbody_debug_level64": (_S, [_P, C.c_int, C.POINTER(_I64), _P, _P]),
     "nbody_get_stats": (_S, [_P, C.POINTER(nbody_stats)]),
     "nbody_direct_accel": (_S, [_P, _P, _I64, _P]),
     "nbody_partition": (_S, [_I64, C.c_int, C.c_int, C.POINTER(_I64), C.POINTER(_I64)]),

@@ -92,6 +92,14 @@ struct nbody_ctx {
   unsigned* xflags = nullptr;       // [kBarrierSlots][kMaxPeers] epochs signalled to this rank
   unsigned* xepoch = nullptr;       // [kBarrierSlots] this rank's barrier counters
   int* xerr = nullptr;              // set by a barrier that timed out
+  // NEXT-2 FP64 mode
+  bool f64 = false;
+  void* arena64 = nullptr;
+  double4* pm64[2] = {nullptr, nullptr};   // pm64[1] = the leaf ids of tree.rec64
+  double4* vi64[2] = {nullptr, nullptr};
+  double4* acc64 = nullptr;
+  double* bbox_part64 = nullptr;
+  double* stage64 = nullptr;               // [n][3] host-transfer staging
   // NEXT-3(i) cost-weighted ranges (peer exchange only)
   bool balance = false;
   uint32_t* gcost = nullptr;        // [ceil(n/32)] interactions per 32-slot group, last pass
@@ -281,6 +289,44 @@ nbody_status allocate(nbody_ctx* c) {
   return NBODY_OK;
 }
 
+// NEXT-2 FP64 mode buffers (one allocation, on first use).
+nbody_status alloc_f64(nbody_ctx* c) {
+  const int64_t n = c->n;
+  const size_t ids = size_t(1) << (c->tree.L + 1), inner = ids / 2;
+  size_t sz[8];
+  int k = 0;
+  sz[k++] = 32 * size_t(n);              // pm64[0]
+  sz[k++] = 32 * size_t(n);              // vi64[0]
+  sz[k++] = 32 * size_t(n);              // vi64[1]
+  sz[k++] = 32 * ids;                    // rec64 (leaf ids = pm64[1])
+  sz[k++] = 32 * inner;                  // blo64
+  sz[k++] = 32 * inner;                  // bhi64
+  sz[k++] = 32 * size_t(n);              // acc64
+  sz[k++] = 48 * size_t(c->nbbox) + 24 * size_t(n);  // bbox partials + staging
+  size_t total = 0;
+  for (int i = 0; i < k; ++i) total += align_up(sz[i]);
+  cudaError_t e = cudaMalloc(&c->arena64, total);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    c->arena64 = nullptr;
+    return fail(c, NBODY_ENOMEM, "FP64 mode buffers (" + std::to_string(total) + " bytes)");
+  }
+  char* p = static_cast<char*>(c->arena64);
+  int i = 0;
+  auto take = [&](void) -> char* { char* r = p; p += align_up(sz[i++]); return r; };
+  c->pm64[0] = (double4*)take();
+  c->vi64[0] = (double4*)take();
+  c->vi64[1] = (double4*)take();
+  double4* rec64 = (double4*)take();
+  c->pm64[1] = rec64 + (int64_t(1) << c->tree.L);
+  c->tree.blo64 = (double4*)take();
+  c->tree.bhi64 = (double4*)take();
+  c->acc64 = (double4*)take();
+  c->bbox_part64 = (double*)take();
+  c->stage64 = c->bbox_part64 + 6 * size_t(c->nbbox);
+  return NBODY_OK;
+}
+
 // NEXT-3(i) is active: peer exchange over G > 1 ranks with balance on.
 bool balanced(const nbody_ctx* c) { return c->balance && c->xpeer && c->world > 1; }
 
@@ -315,13 +361,21 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   const bool tm = c->timing && s == c->stream;
   auto mark = [&](int i) -> cudaError_t { return tm ? cudaEventRecord(c->ev[i], s) : cudaSuccess; };
   CK(mark(0));
-  launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
-  launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
+  const bool f64 = c->f64;
+  if (f64) {  // NEXT-2: fp64 bodies
+    launch_bbox_partial_f64(c->pm64[0], n, c->bbox_part64, c->nbbox, s);
+    launch_bbox_final_f64(c->bbox_part64, c->nbbox, c->b, c->grid, s);
+  } else {
+    launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
+    launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
+  }
   int front_kernels = 2;
   if (resort) {
     CK(cudaMemsetAsync(c->sort.ghist, 0, sizeof(uint32_t) * 8 * 256, s));
     c->sort.hist_ready = true;  // the key kernel fills the sort's digit histograms
-    if (c->key_bytes == 4)
+    if (f64)
+      launch_keys_f64(c->pm64[0], n, c->grid, c->keys[0], c->key_bytes, c->sort.ghist, c->sort.passes, s);
+    else if (c->key_bytes == 4)
       launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), c->sort.ghist, c->sort.passes, s);
     else
       launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), c->sort.ghist,
@@ -332,15 +386,23 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     CK(mark(1));
     c->perm_buf = launch_radix_sort(c->sort, c->keys, c->idx, s);
     CK(mark(2));
-    launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
+    if (f64)
+      launch_permute_f64(c->pm64[0], c->vi64[0], c->idx[c->perm_buf], n, c->pm64[1], c->vi64[1], s);
+    else
+      launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
     front_kernels += 1 + c->sort.passes + 1;
   } else {
     // tree reuse (NEXT-3(iii), [A23]): keep the current (previous Hilbert)
     // order; the leaves are the current state
     CK(mark(1));
     CK(mark(2));
-    CK(cudaMemcpyAsync(c->pm[1], c->pm[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
-    CK(cudaMemcpyAsync(c->vi[1], c->vi[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    if (f64) {
+      CK(cudaMemcpyAsync(c->pm64[1], c->pm64[0], 32 * size_t(n), cudaMemcpyDeviceToDevice, s));
+      CK(cudaMemcpyAsync(c->vi64[1], c->vi64[0], 32 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    } else {
+      CK(cudaMemcpyAsync(c->pm[1], c->pm[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+      CK(cudaMemcpyAsync(c->vi[1], c->vi[0], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    }
   }
   c->last_sorted = resort;
   int x_kernels = 0;
@@ -349,7 +411,10 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     ++x_kernels;
   }
   int build_kernels;
-  if (c->build_variant == 1 && !c->tree.quad) {  // the level-by-level variant is monopole only
+  if (f64) {  // NEXT-2: fp64 leaves at tree.rec64 + 2^L, fp64 boxes
+    launch_build_fused_f64(c->tree, debug, s);
+    build_kernels = c->tree.L < 1 ? 0 : (c->tree.L > 9 ? 2 : 1);
+  } else if (c->build_variant == 1 && !c->tree.quad) {  // the level-by-level variant is monopole only
     launch_build(c->tree, c->pm[1], s);
     build_kernels = c->tree.L;
   } else {
@@ -371,6 +436,11 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   fp.acc = c->acc;
   fp.count = c->cnt;
   fp.total = c->total;
+  if (f64) {  // NEXT-2 (tree.rec64 is set: K6 runs its fp64 variant)
+    fp.leaves64 = c->pm64[1];
+    fp.acc64 = c->acc64;
+    fp.eps2_64 = c->eps * c->eps;
+  }
   const bool bal = balanced(c);
   const int64_t groups = (n + 31) / 32;
   const int64_t cap_groups = std::min(groups, 2 * ((groups + c->world - 1) / c->world));
@@ -393,6 +463,9 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
       launch_partition(c->gcost, groups, c->world, n, cap_groups, c->dpart, c->dpart_used, s);
       ++x_kernels;
     }
+  } else if (integrate && f64) {
+    launch_leapfrog_f64(c->pm64[1] + ob, c->vi64[1] + ob, c->acc64, oe - ob, c->dt, c->pm64[0] + ob,
+                        c->vi64[0] + ob, s);
   } else if (integrate) {
     launch_leapfrog(c->pm[1] + ob, c->vi[1] + ob, c->acc, oe - ob, float(c->dt), c->pm[0] + ob, c->vi[0] + ob, s);
 #ifdef NBODY_WITH_NCCL
@@ -408,6 +481,9 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
         return fail(c, NBODY_ENCCL, ncclGetErrorString(r != ncclSuccess ? r : r2));
     }
 #endif
+  } else if (f64) {
+    CK(cudaMemcpyAsync(c->pm64[0], c->pm64[1], 32 * size_t(n), cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(c->vi64[0], c->vi64[1], 32 * size_t(n), cudaMemcpyDeviceToDevice, s));
   } else {
     CK(cudaMemcpyAsync(c->pm[0], c->pm[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
     CK(cudaMemcpyAsync(c->vi[0], c->vi[1], 16 * size_t(n), cudaMemcpyDeviceToDevice, s));
@@ -570,6 +646,7 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       return NBODY_OK;
     case NBODY_OPT_MULTIPOLE:
       if (value != 1 && value != 2) return fail(c, NBODY_EINVAL, "multipole order must be 1 or 2");
+      if (value == 2 && c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode is monopole only");
       if (value == 2 && !c->tree.S64) {  // allocated on first use: 80 B per internal id
         const size_t inner = size_t(1) << c->tree.L;
         cudaError_t e = cudaMalloc(&c->quad_arena, 48 * inner + 32 * inner);
@@ -592,6 +669,24 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "timing must be 0 or 1");
       c->timing = value != 0;
       return NBODY_OK;
+    case NBODY_OPT_PRECISION: {
+      if (value != 32 && value != 64) return fail(c, NBODY_EINVAL, "precision must be 32 or 64");
+      const bool want = value == 64;
+      if (want && (c->world > 1 || c->xpeer))
+        return fail(c, NBODY_EINVAL, "the FP64 mode runs on a single rank (no exchange)");
+      if (want && (c->tree.quad || c->traversal != 0))
+        return fail(c, NBODY_EINVAL, "the FP64 mode needs monopole order and traversal variant 0");
+      if (want && !c->arena64) {
+        const nbody_status st = alloc_f64(c);
+        if (st != NBODY_OK) return st;
+      }
+      c->f64 = want;
+      c->tree.rec64 = want ? c->pm64[1] - (int64_t(1) << c->tree.L) : nullptr;
+      c->loaded = false;  // bodies must be (re)loaded in the new precision
+      c->have_force = false;
+      drop_graph(c);
+      return NBODY_OK;
+    }
     case NBODY_OPT_BALANCE:
       if (value != 0 && value != 1) return fail(c, NBODY_EINVAL, "balance must be 0 or 1");
       c->balance = value != 0;
@@ -599,6 +694,7 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       return NBODY_OK;
     case NBODY_OPT_TRAVERSAL:
       if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown traversal variant");
+      if (value != 0 && c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode uses traversal variant 0");
       c->traversal = int(value);
       drop_graph(c);
       return NBODY_OK;
@@ -607,8 +703,46 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
   }
 }
 
+nbody_status nbody_set_bodies64(nbody_ctx* c, const double* pos, const double* vel, const double* mass) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "nbody_set_bodies64 needs NBODY_OPT_PRECISION = 64");
+  if (!pos || !vel || !mass) return fail(c, NBODY_EINVAL, "null input");
+  const int64_t n = c->n;
+  const double *dp = pos, *dv = vel, *dm = mass;
+  cudaStream_t s = c->stream;
+  // host inputs go through buffers that the next pass overwrites anyway
+  if (!is_device_ptr(pos)) {
+    CK(cudaMemcpyAsync(c->acc64, pos, 24 * size_t(n), cudaMemcpyDefault, s));
+    dp = reinterpret_cast<const double*>(c->acc64);
+  }
+  if (!is_device_ptr(vel)) {
+    CK(cudaMemcpyAsync(c->pm64[1], vel, 24 * size_t(n), cudaMemcpyDefault, s));
+    dv = reinterpret_cast<const double*>(c->pm64[1]);
+  }
+  if (!is_device_ptr(mass)) {
+    CK(cudaMemcpyAsync(c->vi64[1], mass, 8 * size_t(n), cudaMemcpyDefault, s));
+    dm = reinterpret_cast<const double*>(c->vi64[1]);
+  }
+  CK(cudaMemsetAsync(c->bad, 0, sizeof(int), s));
+  launch_pack_bodies_f64(dp, dv, dm, n, c->pm64[0], c->vi64[0], c->bad, s);
+  CK(cudaGetLastError());
+  int bad = 0;
+  CK(cudaMemcpyAsync(&bad, c->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (bad) {
+    c->loaded = false;
+    return fail(c, NBODY_EINVAL, (bad & 2) ? "masses must be finite and > 0" : "non-finite position or velocity");
+  }
+  c->loaded = true;
+  c->have_force = false;
+  c->keys_dbg_valid = false;
+  c->steps = 0;
+  return NBODY_OK;
+}
+
 nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, const float* mass) {
   CHECK_CTX(c);
+  if (c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: use nbody_set_bodies64");
   if (!pos || !vel || !mass) return fail(c, NBODY_EINVAL, "null input");
   const int64_t n = c->n;
   const float *dp = pos, *dv = vel, *dm = mass;
@@ -714,6 +848,22 @@ static nbody_status get_by_id3(nbody_ctx* c, const float4* src, int64_t b, int64
   return sync_stream(c);
 }
 
+// NEXT-2 FP64 mode: out[id][3] <- src[slot].xyz for all slots (fp64, or
+// rounded to fp32 for the fp32 getters).
+static nbody_status get_by_id3_f64(nbody_ctx* c, const double4* src, void* out, bool as_f32) {
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  const int64_t n = c->n;
+  const bool dev = is_device_ptr(out);
+  void* dst = dev ? out : static_cast<void*>(c->stage64);
+  if (as_f32)
+    launch_scatter_by_id3_f64to32(src, c->vi64[0], n, static_cast<float*>(dst), c->stream);
+  else
+    launch_scatter_by_id3_f64(src, c->vi64[0], n, static_cast<double*>(dst), c->stream);
+  CK(cudaGetLastError());
+  if (!dev) CK(cudaMemcpyAsync(out, dst, (as_f32 ? 12 : 24) * size_t(n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
 #ifdef NBODY_WITH_NCCL
 // Collective: gather every rank's owned slice of src (S records of `words`
 // 4-byte words) into dst, indexed by slot.
@@ -727,6 +877,7 @@ static nbody_status gather_owned(nbody_ctx* c, const void* src, void* dst, size_
 nbody_status nbody_get_accel(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  if (c->f64) return get_by_id3_f64(c, c->acc64, out, true);
 #ifdef NBODY_WITH_NCCL
   if (c->comm) {
     nbody_status s = gather_owned(c, c->acc, c->stage, 4);
@@ -745,13 +896,36 @@ nbody_status nbody_get_accel(nbody_ctx* c, float* out) {
 nbody_status nbody_get_positions(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (c->f64) return get_by_id3_f64(c, c->pm64[0], out, true);
   return get_by_id3(c, c->pm[0], 0, c->n, out);
 }
 
 nbody_status nbody_get_velocities(nbody_ctx* c, float* out) {
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (c->f64) return get_by_id3_f64(c, c->vi64[0], out, true);
   return get_by_id3(c, c->vi[0], 0, c->n, out);
+}
+
+nbody_status nbody_get_positions64(nbody_ctx* c, double* out) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "needs NBODY_OPT_PRECISION = 64");
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  return get_by_id3_f64(c, c->pm64[0], out, false);
+}
+
+nbody_status nbody_get_velocities64(nbody_ctx* c, double* out) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "needs NBODY_OPT_PRECISION = 64");
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  return get_by_id3_f64(c, c->vi64[0], out, false);
+}
+
+nbody_status nbody_get_accel64(nbody_ctx* c, double* out) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "needs NBODY_OPT_PRECISION = 64");
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  return get_by_id3_f64(c, c->acc64, out, false);
 }
 
 nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
@@ -780,7 +954,10 @@ nbody_status nbody_get_interactions(nbody_ctx* c, uint32_t* out) {
   const bool dev = is_device_ptr(out);
   uint32_t* dst = dev ? out : reinterpret_cast<uint32_t*>(c->out3);
   if (!dev && (b > 0 || e < n)) CK(cudaMemcpyAsync(dst, out, 4 * size_t(n), cudaMemcpyDefault, c->stream));
-  launch_scatter_by_id1(src, c->vi[0] + b, e - b, dst, c->stream);
+  if (c->f64)
+    launch_scatter_by_id1_f64(src, c->vi64[0] + b, e - b, dst, c->stream);
+  else
+    launch_scatter_by_id1(src, c->vi[0] + b, e - b, dst, c->stream);
   CK(cudaGetLastError());
   if (!dev) CK(cudaMemcpyAsync(out, dst, 4 * size_t(n), cudaMemcpyDefault, c->stream));
   return sync_stream(c);
@@ -792,6 +969,7 @@ nbody_status nbody_direct_accel(nbody_ctx* c, const int64_t* ids, int64_t nt, do
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
   if (nt < 0 || (nt > 0 && (!ids || !out))) return fail(c, NBODY_EINVAL, "bad target list");
+  if (c->f64) return fail(c, NBODY_EINVAL, "nbody_direct_accel works on the fp32 state (precision 32)");
   if (nt == 0) return NBODY_OK;
   const bool ids_dev = is_device_ptr(ids);
   if (!ids_dev)
@@ -824,6 +1002,7 @@ nbody_status nbody_set_partition(nbody_ctx* c, int rank, int world) {
   CHECK_CTX(c);
   if (world < 1 || world > kMaxWorld || rank < 0 || rank >= world)
     return fail(c, NBODY_EINVAL, "need 0 <= rank < world <= 256");
+  if (c->f64 && world > 1) return fail(c, NBODY_EINVAL, "the FP64 mode runs on a single rank");
 #ifdef NBODY_WITH_NCCL
   if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is attached");
 #endif
@@ -893,6 +1072,7 @@ nbody_status nbody_attach_nccl(nbody_ctx* c, const void* unique_id, int rank, in
   CHECK_CTX(c);
   if (!unique_id || world < 1 || world > kMaxWorld || rank < 0 || rank >= world)
     return fail(c, NBODY_EINVAL, "need a unique id and 0 <= rank < world <= 256");
+  if (c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode runs on a single rank");
 #ifdef NBODY_WITH_NCCL
   if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is already attached");
   if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are attached");
@@ -927,6 +1107,7 @@ nbody_status nbody_peer_handle(nbody_ctx* c, void* out) {
 }
 
 static nbody_status check_attach(nbody_ctx* c, int rank, int world) {
+  if (c && c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode runs on a single rank");
   if (world < 1 || world > kMaxPeers || rank < 0 || rank >= world)
     return fail(c, NBODY_EINVAL, "peer exchange needs 0 <= rank < world <= 8");
   if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are already attached");
@@ -1003,8 +1184,18 @@ int nbody_exchange_mode(nbody_ctx* c) {
   return 0;
 }
 
+nbody_status nbody_get_state64(nbody_ctx* c, double* pos_m, double* vel_id) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "needs NBODY_OPT_PRECISION = 64");
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (pos_m) CK(cudaMemcpyAsync(pos_m, c->pm64[0], 32 * size_t(c->n), cudaMemcpyDefault, c->stream));
+  if (vel_id) CK(cudaMemcpyAsync(vel_id, c->vi64[0], 32 * size_t(c->n), cudaMemcpyDefault, c->stream));
+  return sync_stream(c);
+}
+
 nbody_status nbody_get_state(nbody_ctx* c, float* pos_m, float* vel_id) {
   CHECK_CTX(c);
+  if (c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: use nbody_get_state64");
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
   if (pos_m) CK(cudaMemcpyAsync(pos_m, c->pm[0], 16 * size_t(c->n), cudaMemcpyDefault, c->stream));
   if (vel_id) CK(cudaMemcpyAsync(vel_id, c->vi[0], 16 * size_t(c->n), cudaMemcpyDefault, c->stream));
@@ -1107,9 +1298,28 @@ nbody_status nbody_debug_level(nbody_ctx* c, int level, int64_t* count, double* 
   cudaStream_t s = c->stream;
   if (pred) CK(cudaMemcpyAsync(pred, c->tree.pred + off, 32 * size_t(cnt), cudaMemcpyDefault, s));
   if (rec) CK(cudaMemcpyAsync(rec, c->tree.rec + off, 16 * size_t(cnt), cudaMemcpyDefault, s));
+  if (box && c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: fp64 boxes via nbody_debug_level64");
   if (box) {
     CK(cudaMemcpy2DAsync(box, 24, c->tree.blo + off, 16, 12, size_t(cnt), cudaMemcpyDefault, s));
     CK(cudaMemcpy2DAsync(box + 3, 24, c->tree.bhi + off, 16, 12, size_t(cnt), cudaMemcpyDefault, s));
+  }
+  return sync_stream(c);
+}
+
+nbody_status nbody_debug_level64(nbody_ctx* c, int level, int64_t* count, double* rec64, double* box64) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "needs NBODY_OPT_PRECISION = 64");
+  if (level < 1 || level > c->tree.L) return fail(c, NBODY_EINVAL, "level out of range [1, L]");
+  const int64_t cnt = c->tree.count[level];
+  if (count) *count = cnt;
+  if (!rec64 && !box64) return NBODY_OK;
+  if (!c->have_force) return fail(c, NBODY_ESTATE, "no force pass yet");
+  const int64_t off = c->tree.off[level];
+  cudaStream_t s = c->stream;
+  if (rec64) CK(cudaMemcpyAsync(rec64, c->tree.rec64 + off, 32 * size_t(cnt), cudaMemcpyDefault, s));
+  if (box64) {
+    CK(cudaMemcpy2DAsync(box64, 48, c->tree.blo64 + off, 32, 24, size_t(cnt), cudaMemcpyDefault, s));
+    CK(cudaMemcpy2DAsync(box64 + 3, 48, c->tree.bhi64 + off, 32, 24, size_t(cnt), cudaMemcpyDefault, s));
   }
   return sync_stream(c);
 }
@@ -1130,6 +1340,7 @@ void nbody_destroy(nbody_ctx* c) {
     if (p) cudaIpcCloseMemHandle(p);
   if (c->arena) cudaFree(c->arena);
   if (c->quad_arena) cudaFree(c->quad_arena);
+  if (c->arena64) cudaFree(c->arena64);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
   if (c->cap_stream) cudaStreamDestroy(c->cap_stream);

@@ -22,6 +22,8 @@ struct GridInfo {
   float abs_d2;  // absolute slack of the fp32 opening-test filter: 1e-9 R^2,
                  // R = max |coordinate| (K6)
   float R;       // max |coordinate| of this step's bodies (T-filter slack)
+  double lo64[3];  // NEXT-2 FP64 mode: the fp64 bounding box (lo/hi unused)
+  double hi64[3];
 };
 
 // NEXT-4 [A24]: second mass moment about the COM, S = sum m (x-c)(x-c)^T.
@@ -47,6 +49,10 @@ struct TreeView {
   const GridInfo* grid;  // bbox of this step (filter slack)
   double th2;            // theta^2 the thresholds were built for
   double4* mom;    // (M, Mx, My, Mz) fp64 moments (build only) [A12]
+  double4* rec64 = nullptr;  // NEXT-2 FP64 mode, every id: (com64, M) of an
+                             // internal node, the sorted body (x, m) at a leaf
+  double4* blo64 = nullptr;  // NEXT-2 FP64 mode: fp64 AABB (build only)
+  double4* bhi64 = nullptr;
   float4* blo;     // AABB lo (x, y, z, -)
   float4* bhi;     // AABB hi (x, y, z, -)
   bool quad;       // NEXT-4: build second moments, add quadrupole terms
@@ -75,7 +81,11 @@ struct ForceParams {
   int64_t t_end;
   double th2;             // theta^2 (fp64, used by the opening test)
   float eps2;             // eps^2 (fp32 interaction)
+  double eps2_64 = 0.0;   // eps^2 (fp64 interaction, NEXT-2 FP64 mode)
   float4* acc;            // per owned slot (ax, ay, az, 0), indexed slot - t_begin
+  // NEXT-2 FP64 mode (t.rec64 set): targets from leaves64, results to acc64
+  const double4* leaves64 = nullptr;
+  double4* acc64 = nullptr;
   uint32_t* count;        // interactions per owned slot
   unsigned long long* total;  // sum of interactions (integer atomics only)
   // NEXT-3(i) cost-weighted ranges: when part != null the owned range is
@@ -96,6 +106,12 @@ void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* key
                    cudaStream_t s);
 void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
                    int passes, cudaStream_t s);
+// NEXT-2 FP64 mode: the same stages on fp64 bodies (x, y, z, m) as double4;
+// partial[block][6] doubles; the grid's lo64/hi64 hold the box.
+void launch_bbox_partial_f64(const double4* pm, int64_t n, double* partial, int nblocks, cudaStream_t s);
+void launch_bbox_final_f64(const double* partial, int nparts, int b, GridInfo* g, cudaStream_t s);
+void launch_keys_f64(const double4* pm, int64_t n, const GridInfo* g, void* keys, int key_bytes, uint32_t* ghist,
+                     int passes, cudaStream_t s);
 
 // ---- K3 radix sort ---------------------------------------------------------
 struct SortPlan {
@@ -121,6 +137,10 @@ void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);  // 
 // levels 1..10 fused per 1024-leaf subtree + one block for the top levels;
 // keep_all also stores every node's moments/box (debug views)
 void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, cudaStream_t s);
+// NEXT-2 FP64 mode: leaves are t.rec64 + 2^L (fp64 bodies); boxes in fp64
+void launch_permute_f64(const double4* pm_in, const double4* vi_in, const uint32_t* perm, int64_t n,
+                        double4* pm_out, double4* vi_out, cudaStream_t s);
+void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s);
 
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
@@ -142,6 +162,14 @@ void launch_pack_bodies(const float* pos, const float* vel, const float* mass, i
 // out[id][3] <- src[slot].xyz for slots [0, n); id from vi[slot].w
 void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s);
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s);
+// NEXT-2 FP64 mode helpers: ids are vi.w (exact integers in fp64)
+void launch_leapfrog_f64(const double4* pm_in, const double4* vi_in, const double4* acc, int64_t n, double dt,
+                         double4* pm_out, double4* vi_out, cudaStream_t s);
+void launch_pack_bodies_f64(const double* pos, const double* vel, const double* mass, int64_t n, double4* pm,
+                            double4* vi, int* bad, cudaStream_t s);
+void launch_scatter_by_id3_f64(const double4* src, const double4* vi, int64_t n, double* out, cudaStream_t s);
+void launch_scatter_by_id3_f64to32(const double4* src, const double4* vi, int64_t n, float* out, cudaStream_t s);
+void launch_scatter_by_id1_f64(const uint32_t* src, const double4* vi, int64_t n, uint32_t* out, cudaStream_t s);
 
 // ---- K7 fused with the exchange over peer memory -------------
 // Leapfrog of the owned slots [b, b + len) (acc indexed from 0), storing the

@@ -86,6 +86,79 @@ __global__ void k_bbox_final(const float* __restrict__ partial, int nparts, int 
   }
 }
 
+// NEXT-2 FP64 mode: the same reductions on fp64 bodies (exact min/max).
+__device__ __forceinline__ double warp_min_d(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ double warp_max_d(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+__global__ __launch_bounds__(kBBoxThreads) void k_bbox_partial_f64(const double4* __restrict__ pm, int64_t n,
+                                                                   double* __restrict__ partial) {
+  double lo[3] = {DBL_MAX, DBL_MAX, DBL_MAX}, hi[3] = {-DBL_MAX, -DBL_MAX, -DBL_MAX};
+  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const double4 p = pm[i];
+    lo[0] = fmin(lo[0], p.x); hi[0] = fmax(hi[0], p.x);
+    lo[1] = fmin(lo[1], p.y); hi[1] = fmax(hi[1], p.y);
+    lo[2] = fmin(lo[2], p.z); hi[2] = fmax(hi[2], p.z);
+  }
+  __shared__ double s[kBBoxThreads / 32][6];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int k = 0; k < 3; ++k) {
+    lo[k] = warp_min_d(lo[k]);
+    hi[k] = warp_max_d(hi[k]);
+  }
+  if (lane == 0)
+    for (int k = 0; k < 3; ++k) {
+      s[w][k] = lo[k];
+      s[w][3 + k] = hi[k];
+    }
+  __syncthreads();
+  if (threadIdx.x < 6) {
+    const int c = threadIdx.x;
+    double v = s[0][c];
+    for (int k = 1; k < kBBoxThreads / 32; ++k) v = c < 3 ? fmin(v, s[k][c]) : fmax(v, s[k][c]);
+    partial[6 * blockIdx.x + c] = v;
+  }
+}
+
+// ext = max_k (hi_k - lo_k) rounded in fp64 (the oracle's expression on fp64
+// bodies), inv = 2^b / ext; R = max |coordinate| rounded up to fp32; the
+// fp32 filter slack covers the extra rounding of x to fp32 (4e-9 R^2 >
+// 1e-9 R^2 + the 2uR|d| cross term).
+__global__ void k_bbox_final_f64(const double* __restrict__ partial, int nparts, int b, GridInfo* __restrict__ g) {
+  __shared__ double s[6];
+  const int c = threadIdx.x;
+  if (c < 6) {
+    double v = partial[c];
+    for (int k = 1; k < nparts; ++k) v = c < 3 ? fmin(v, partial[6 * k + c]) : fmax(v, partial[6 * k + c]);
+    s[c] = v;
+  }
+  __syncthreads();
+  if (c == 0) {
+    double ext = 0.0, R = 0.0;
+    for (int k = 0; k < 3; ++k) {
+      g->lo64[k] = s[k];
+      g->hi64[k] = s[3 + k];
+      g->lo[k] = __double2float_rd(s[k]);
+      g->hi[k] = __double2float_ru(s[3 + k]);
+      ext = fmax(ext, __dsub_rn(s[3 + k], s[k]));
+      R = fmax(R, fmax(fabs(s[k]), fabs(s[3 + k])));
+    }
+    g->inv = ext > 0.0 ? __ddiv_rn(double(1u << b), ext) : 0.0;
+    g->b = b;
+    const float Rf = __double2float_ru(R);
+    g->abs_d2 = fmaxf(4e-9f * Rf * Rf, 1e-37f);
+    g->R = Rf;
+  }
+}
+
 // Spread the low 21 bits of v so that bit q lands at bit 3q.
 __device__ __forceinline__ unsigned long long spread3(uint32_t v) {
   unsigned long long x = v & 0x1fffffull;
@@ -131,10 +204,11 @@ constexpr int kKeysThreads = 256;
 // sort passes).  Grid-stride; per-block shared histograms; a warp whose 32
 // keys share a digit adds it once (common for the high digits: the input is
 // the previous step's Hilbert order).
-template <class K>
-__global__ __launch_bounds__(kKeysThreads) void k_keys(const float4* __restrict__ pm, int64_t n,
+template <class K, class V4>
+__global__ __launch_bounds__(kKeysThreads) void k_keys(const V4* __restrict__ pm, int64_t n,
                                                        const GridInfo* __restrict__ gi, K* __restrict__ keys,
                                                        uint32_t* __restrict__ ghist, int passes) {
+  constexpr bool kF64 = sizeof(V4) == 32;  // NEXT-2: fp64 bodies, fp64 box
   __shared__ uint32_t sh[8 * 256];
   for (int i = threadIdx.x; i < passes * 256; i += kKeysThreads) sh[i] = 0;
   __syncthreads();
@@ -147,12 +221,14 @@ __global__ __launch_bounds__(kKeysThreads) void k_keys(const float4* __restrict_
     const bool ok = i < n;
     K key = 0;
     if (ok) {
-      const float4 p = __ldg(pm + i);
+      const V4 p = pm[i];
+      const double l0 = kF64 ? g.lo64[0] : double(g.lo[0]), l1 = kF64 ? g.lo64[1] : double(g.lo[1]),
+                   l2 = kF64 ? g.lo64[2] : double(g.lo[2]);
       // q_k = min(2^b - 1, floor((x_k - lo_k) * inv)) in fp64; the operand is
       // >= 0, so truncation is the floor.
-      const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), double(g.lo[0])), g.inv)));
-      const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), double(g.lo[1])), g.inv)));
-      const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), double(g.lo[2])), g.inv)));
+      const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), l0), g.inv)));
+      const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), l1), g.inv)));
+      const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), l2), g.inv)));
       key = K(hilbert3(q0, q1, q2, g.b));
       keys[i] = key;
     }
@@ -196,6 +272,23 @@ void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* key
 void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
                    int passes, cudaStream_t s) {
   k_keys<unsigned long long><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
+}
+
+void launch_bbox_partial_f64(const double4* pm, int64_t n, double* partial, int nblocks, cudaStream_t s) {
+  k_bbox_partial_f64<<<nblocks, kBBoxThreads, 0, s>>>(pm, n, partial);
+}
+
+void launch_bbox_final_f64(const double* partial, int nparts, int b, GridInfo* g, cudaStream_t s) {
+  k_bbox_final_f64<<<1, 32, 0, s>>>(partial, nparts, b, g);
+}
+
+void launch_keys_f64(const double4* pm, int64_t n, const GridInfo* g, void* keys, int key_bytes, uint32_t* ghist,
+                     int passes, cudaStream_t s) {
+  if (key_bytes == 4)
+    k_keys<uint32_t><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, static_cast<uint32_t*>(keys), ghist, passes);
+  else
+    k_keys<unsigned long long>
+        <<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, static_cast<unsigned long long*>(keys), ghist, passes);
 }
 
 }  // namespace nb

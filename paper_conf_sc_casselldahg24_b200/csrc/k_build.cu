@@ -14,6 +14,8 @@
 // Default variant: a block reduces a 1024-leaf subtree (levels 1..10) in
 // shared memory and one block builds the top levels; variant 1 launches one
 // kernel per level (monopole only).  Both give identical records.
+#include <type_traits>
+
 #include "internal.cuh"
 
 namespace nb {
@@ -38,18 +40,48 @@ __device__ __forceinline__ void add_second_moment(double* Sp, const double* Sc, 
   for (int q = 0; q < 6; ++q) Sp[q] = __dadd_rn(Sp[q], __dadd_rn(Sc[q], __dmul_rn(__dmul_rn(Mc, di[q]), dj[q])));
 }
 
+// Box helpers for fp32 (float4) and fp64 (double4, NEXT-2) bounds: exact
+// min/max either way.
+__device__ __forceinline__ float4 box_min(float4 a, float4 b) {
+  return make_float4(fminf(a.x, b.x), fminf(a.y, b.y), fminf(a.z, b.z), 0.f);
+}
+__device__ __forceinline__ float4 box_max(float4 a, float4 b) {
+  return make_float4(fmaxf(a.x, b.x), fmaxf(a.y, b.y), fmaxf(a.z, b.z), 0.f);
+}
+__device__ __forceinline__ double4 box_min(double4 a, double4 b) {
+  return make_double4(fmin(a.x, b.x), fmin(a.y, b.y), fmin(a.z, b.z), 0.0);
+}
+__device__ __forceinline__ double4 box_max(double4 a, double4 b) {
+  return make_double4(fmax(a.x, b.x), fmax(a.y, b.y), fmax(a.z, b.z), 0.0);
+}
+__device__ __forceinline__ void store_box(const TreeView& t, int64_t node, float4 lo, float4 hi) {
+  t.blo[node] = lo;
+  t.bhi[node] = hi;
+}
+__device__ __forceinline__ void store_box(const TreeView& t, int64_t node, double4 lo, double4 hi) {
+  t.blo64[node] = lo;
+  t.bhi64[node] = hi;
+}
+__device__ __forceinline__ float4 load_lo(const TreeView& t, int64_t node, float4*) { return t.blo[node]; }
+__device__ __forceinline__ float4 load_hi(const TreeView& t, int64_t node, float4*) { return t.bhi[node]; }
+__device__ __forceinline__ double4 load_lo(const TreeView& t, int64_t node, double4*) { return t.blo64[node]; }
+__device__ __forceinline__ double4 load_hi(const TreeView& t, int64_t node, double4*) { return t.bhi64[node]; }
+
 // Emit node `node` with centre of mass c: the traversal records (pred, rec,
-// rc[, qf]) always; the build moments, box [and S64] only when `keep`
-// (needed by a parent built in another block, or by the debug views).
+// rc, tf[, qf][, rec64]) always; the build moments, box [and S64] only when
+// `keep` (needed by a parent built in another block, or by the debug views).
+template <class B4>
 __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, double M, double mx, double my, double mz,
-                                            const double* c, float4 lo, float4 hi, bool keep,
+                                            const double* c, B4 lo, B4 hi, bool keep,
                                             const double* S = nullptr) {
+  constexpr bool kF64 = sizeof(B4) == 32;
   if (keep) {
     t.mom[node] = make_double4(M, mx, my, mz);
-    t.blo[node] = lo;
-    t.bhi[node] = hi;
+    store_box(t, node, lo, hi);
   }
-  // [A3] s = longest side of the AABB (fp64 differences of fp32 bounds are exact)
+  if (kF64) t.rec64[node] = make_double4(c[0], c[1], c[2], M);
+  // [A3] s = longest side of the AABB (fp64 differences: exact for fp32
+  // bounds, rounded for fp64 bounds -- the oracle's expression either way)
   double s = __dsub_rn(double(hi.x), double(lo.x));
   s = fmax(s, __dsub_rn(double(hi.y), double(lo.y)));
   s = fmax(s, __dsub_rn(double(hi.z), double(lo.z)));
@@ -158,35 +190,40 @@ constexpr int fuse_half() {  // level-1 nodes per block (quad: 512-leaf subtrees
   return kQuad ? kFuseHalf / 2 : kFuseHalf;
 }
 
-template <bool kQuad>
+template <bool kQuad, bool kF64>
 __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const float4* __restrict__ leaves, int top,
                                                               bool keep_all) {
-  constexpr int kHalf = kQuad ? kFuseHalf / 2 : kFuseHalf;
+  using B4 = typename std::conditional<kF64, double4, float4>::type;  // box / leaf type
+  constexpr int kHalf = (kQuad || kF64) ? kFuseHalf / 2 : kFuseHalf;
   __shared__ double4 s_m[kHalf];
-  __shared__ float4 s_lo[kHalf];
-  __shared__ float4 s_hi[kHalf];
+  __shared__ B4 s_lo[kHalf];
+  __shared__ B4 s_hi[kHalf];
   __shared__ double s_c[kQuad ? 3 * kHalf : 1];
   __shared__ double s_S[kQuad ? 6 * kHalf : 1];
+  const B4* lv = kF64 ? reinterpret_cast<const B4*>(t.rec64 + (int64_t(1) << t.L))
+                      : reinterpret_cast<const B4*>(leaves);
   const int64_t b = blockIdx.x;
   for (int q = threadIdx.x; q < kHalf; q += kFuseThreads) {
     const int64_t j = b * kHalf + q;
     if (j >= t.count[1]) continue;
     const int64_t a = 2 * j;
-    const float4 A = __ldg(leaves + a);
+    const B4 A = lv[a];
     const bool two = a + 1 < t.n;
-    const float4 B = two ? __ldg(leaves + a + 1) : A;
+    const B4 B = two ? lv[a + 1] : A;
     double M = double(A.w);
     double mx = __dmul_rn(double(A.w), double(A.x));
     double my = __dmul_rn(double(A.w), double(A.y));
     double mz = __dmul_rn(double(A.w), double(A.z));
-    float4 lo = make_float4(A.x, A.y, A.z, 0.f), hi = lo;
+    B4 lo = A, hi = A;
+    lo.w = 0;
+    hi.w = 0;
     if (two) {
       M = __dadd_rn(M, double(B.w));
       mx = __dadd_rn(mx, __dmul_rn(double(B.w), double(B.x)));
       my = __dadd_rn(my, __dmul_rn(double(B.w), double(B.y)));
       mz = __dadd_rn(mz, __dmul_rn(double(B.w), double(B.z)));
-      lo.x = fminf(lo.x, B.x); lo.y = fminf(lo.y, B.y); lo.z = fminf(lo.z, B.z);
-      hi.x = fmaxf(hi.x, B.x); hi.y = fmaxf(hi.y, B.y); hi.z = fmaxf(hi.z, B.z);
+      lo = box_min(lo, B);
+      hi = box_max(hi, B);
     }
     double c[3];
     node_com(M, mx, my, mz, c);
@@ -218,7 +255,7 @@ __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const 
     const int64_t j = b * cnt + q;
     bool have = false;
     double4 m;
-    float4 lo, hi;
+    B4 lo, hi;
     double c[3], S[6];
     if (q < cnt && j < t.count[l]) {
       have = true;
@@ -228,13 +265,12 @@ __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const 
       hi = s_hi[2 * q];
       if (two) {
         const double4 mb = s_m[2 * q + 1];
-        const float4 lb = s_lo[2 * q + 1], hb = s_hi[2 * q + 1];
         m.x = __dadd_rn(m.x, mb.x);
         m.y = __dadd_rn(m.y, mb.y);
         m.z = __dadd_rn(m.z, mb.z);
         m.w = __dadd_rn(m.w, mb.w);
-        lo.x = fminf(lo.x, lb.x); lo.y = fminf(lo.y, lb.y); lo.z = fminf(lo.z, lb.z);
-        hi.x = fmaxf(hi.x, hb.x); hi.y = fmaxf(hi.y, hb.y); hi.z = fmaxf(hi.z, hb.z);
+        lo = box_min(lo, s_lo[2 * q + 1]);
+        hi = box_max(hi, s_hi[2 * q + 1]);
       }
       node_com(m.x, m.y, m.z, m.w, c);
       if (kQuad) {
@@ -263,22 +299,24 @@ __global__ __launch_bounds__(kFuseThreads) void k_build_fused(TreeView t, const 
 
 // Levels from..L in one block (the top of the tree is small: ceil(N / 2^l)
 // nodes per level); __syncthreads orders the levels.
+template <bool kF64>
 __global__ __launch_bounds__(1024) void k_build_upper(TreeView t, int from) {
+  using B4 = typename std::conditional<kF64, double4, float4>::type;
+  B4* tag = nullptr;
   for (int l = from; l <= t.L; ++l) {
     for (int64_t j = threadIdx.x; j < t.count[l]; j += blockDim.x) {
       const int64_t ca = t.off[l - 1] + 2 * j;
       const bool two = 2 * j + 1 < t.count[l - 1];
       double4 m = t.mom[ca];
-      float4 lo = t.blo[ca], hi = t.bhi[ca];
+      B4 lo = load_lo(t, ca, tag), hi = load_hi(t, ca, tag);
       if (two) {
         const double4 mb = t.mom[ca + 1];
-        const float4 lb = t.blo[ca + 1], hb = t.bhi[ca + 1];
         m.x = __dadd_rn(m.x, mb.x);
         m.y = __dadd_rn(m.y, mb.y);
         m.z = __dadd_rn(m.z, mb.z);
         m.w = __dadd_rn(m.w, mb.w);
-        lo.x = fminf(lo.x, lb.x); lo.y = fminf(lo.y, lb.y); lo.z = fminf(lo.z, lb.z);
-        hi.x = fmaxf(hi.x, hb.x); hi.y = fmaxf(hi.y, hb.y); hi.z = fmaxf(hi.z, hb.z);
+        lo = box_min(lo, load_lo(t, ca + 1, tag));
+        hi = box_max(hi, load_hi(t, ca + 1, tag));
       }
       double c[3];
       node_com(m.x, m.y, m.z, m.w, c);
@@ -301,6 +339,17 @@ __global__ __launch_bounds__(1024) void k_build_upper(TreeView t, int from) {
   }
 }
 
+__global__ __launch_bounds__(256) void k_permute_f64(const double4* __restrict__ pm_in,
+                                                     const double4* __restrict__ vi_in,
+                                                     const uint32_t* __restrict__ perm, int64_t n,
+                                                     double4* __restrict__ pm_out, double4* __restrict__ vi_out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t p = perm[i];
+  pm_out[i] = pm_in[p];
+  vi_out[i] = vi_in[p];
+}
+
 }  // namespace
 
 void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, cudaStream_t s) {
@@ -310,10 +359,25 @@ void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, 
   const int top = t.L < levels ? t.L : levels;
   const unsigned grid = unsigned((t.count[1] + half - 1) / half);
   if (t.quad)
-    k_build_fused<true><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
+    k_build_fused<true, false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
   else
-    k_build_fused<false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
-  if (t.L > top) k_build_upper<<<1, 1024, 0, s>>>(t, top + 1);
+    k_build_fused<false, false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
+  if (t.L > top) k_build_upper<false><<<1, 1024, 0, s>>>(t, top + 1);
+}
+
+void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s) {
+  if (t.L < 1) return;
+  const int levels = kFuseLevels - 1;  // 512-leaf subtrees (fp64 boxes in shared memory)
+  const int half = kFuseHalf / 2;
+  const int top = t.L < levels ? t.L : levels;
+  const unsigned grid = unsigned((t.count[1] + half - 1) / half);
+  k_build_fused<false, true><<<grid, kFuseThreads, 0, s>>>(t, nullptr, top, keep_all);
+  if (t.L > top) k_build_upper<true><<<1, 1024, 0, s>>>(t, top + 1);
+}
+
+void launch_permute_f64(const double4* pm_in, const double4* vi_in, const uint32_t* perm, int64_t n,
+                        double4* pm_out, double4* vi_out, cudaStream_t s) {
+  k_permute_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm_in, vi_in, perm, n, pm_out, vi_out);
 }
 
 void launch_permute(const float4* pm_in, const float4* vi_in, const uint32_t* perm, int64_t n, float4* pm_out,

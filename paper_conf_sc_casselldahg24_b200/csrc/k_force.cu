@@ -48,6 +48,8 @@
 // Per-lane opening decisions use an fp32 filter with a rigorous error bound
 // and fall back to the exact fp64 expression inside the uncertainty band
 // (DESIGN.md "fp32 filter"), so they equal the fp64 decisions.
+#include <type_traits>
+
 #include "internal.cuh"
 
 namespace nb {
@@ -103,9 +105,11 @@ __device__ __forceinline__ bool opening_accept64(const double4& p, double x, dou
 }
 
 struct Target {
-  float x, y, z;    // the lane's target position
+  float x, y, z;    // the lane's target position (fp32; rounded in FP64 mode)
   float eps2;
   double th2;
+  double x64 = 0.0, y64 = 0.0, z64 = 0.0;  // NEXT-2 FP64 mode: the exact position
+  double eps2_64 = 0.0;
 };
 
 struct Acc {
@@ -121,6 +125,26 @@ struct Acc {
     z = fmaf(w, dz, z);
   }
 };
+
+// NEXT-2 FP64 mode accumulator and interaction (the paper's precision,
+// P:272): a += m r / (|r|^2 + eps^2)^(3/2), r = s - x, all in fp64; r2 == 0
+// (eps = 0, coincident) adds exactly 0 [A1].
+struct AccD {
+  double x = 0.0, y = 0.0, z = 0.0;
+  uint32_t n = 0;
+};
+
+template <bool kSoft>
+__device__ __forceinline__ void interact64(AccD& a, const double4& s, double m, const Target& T) {
+  const double dx = s.x - T.x64, dy = s.y - T.y64, dz = s.z - T.z64;
+  const double r2 = fma(dz, dz, fma(dy, dy, fma(dx, dx, T.eps2_64)));
+  double inv = rsqrt(r2);
+  if (!kSoft) inv = r2 > 0.0 ? inv : 0.0;
+  const double w = (m * inv) * (inv * inv);
+  a.x = fma(w, dx, a.x);
+  a.y = fma(w, dy, a.y);
+  a.z = fma(w, dz, a.z);
+}
 
 // NEXT-4 [A24]: the quadrupole term of internal node qid (the oracle's
 // interact_quad in fp32): with d = com - x, inv = (|d|^2 + eps^2)^(-1/2),
@@ -162,6 +186,7 @@ struct Walk {
   const float4* rc2;     // rc viewed as pairs (lo_A, hi_A, lo_B, hi_B)
   const float2* rc;
   const double4* pred;
+  const double4* rec64;  // NEXT-2 FP64 mode records (or null)
   const float4* qf;      // NEXT-4 quadrupoles (2 float4 per id) or null
   uint32_t leaf0, n;
   int L;
@@ -179,6 +204,7 @@ __device__ __forceinline__ Walk make_walk(const ForceParams& P) {
   W.rc = in_reg(P.t.rc);
   W.rc2 = reinterpret_cast<const float4*>(W.rc);
   W.pred = in_reg(P.t.pred);
+  W.rec64 = P.t.rec64;
   W.qf = P.t.qf;
   W.L = P.t.L;
   W.leaf0 = 1u << W.L;
@@ -191,9 +217,24 @@ __device__ __forceinline__ bool decide1(const Walk& W, uint32_t g, bool in, floa
   bool acc = in && d2 > c.y;
   const bool und = in && !acc && !(d2 < c.x);
   if (__any_sync(kFull, und)) {
-    if (und) acc = opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
+    if (und) acc = W.rec64 ? opening_accept64(W.pred[g], T.x64, T.y64, T.z64, T.th2)
+                           : opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
   }
   return acc;
+}
+
+// One mask-walk interaction with record r (fp32) / node id g (FP64 mode:
+// the fp64 record rec64[g]).
+__device__ __forceinline__ void walk_add(Acc& a, bool on, const Probe& p, const float4& r, const Walk&, uint32_t,
+                                         const Target& T) {
+  a.add(on, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+}
+__device__ __forceinline__ void walk_add(AccD& a, bool on, const Probe&, const float4&, const Walk& W, uint32_t g,
+                                         const Target& T) {
+  if (on) {
+    const double4 s = W.rec64[g];
+    interact64<false>(a, s, s.w, T);
+  }
 }
 
 // The per-lane mask-stack walk of the subtree of node g0 for the lanes in
@@ -205,8 +246,8 @@ __device__ __forceinline__ void quad_at(Acc& a, const Probe& p, float eps2, cons
   quad_term(a, p.dx, p.dy, p.dz, inv, qf, g, on);
 }
 
-template <bool kQuad>
-__device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32_t kid, Acc& a, int lane, uint32_t g0,
+template <bool kQuad, class AccT>
+__device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32_t kid, AccT& a, int lane, uint32_t g0,
                                           uint32_t mask0) {
   // the start node on its own
   {
@@ -215,14 +256,14 @@ __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32
     const Probe p = probe(r, T);
     if (g0 >= W.leaf0) {  // a leaf (N == 1 root)
       const bool acc = in && g0 != kid;
-      a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
+      walk_add(a, acc, p, r, W, g0, T);
       a.n += acc;
       return;
     }
     const bool acc = decide1(W, g0, in, p.d2, __ldg(W.rc + g0), T);
     if (__any_sync(kFull, acc)) {
-      a.add(acc, p.dx, p.dy, p.dz, p.d2, r.w, T.eps2);
-      if (kQuad) quad_at(a, p, T.eps2, W.qf, g0, acc);
+      walk_add(a, acc, p, r, W, g0, T);
+      if constexpr (kQuad) quad_at(a, p, T.eps2, W.qf, g0, acc);
     }
     a.n += acc;
     const uint32_t rej = __ballot_sync(kFull, in && !acc);
@@ -255,8 +296,10 @@ __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32
       const bool undA = in && !accA && !(pA.d2 < c.x);
       const bool undB = in && hasB && !accB && !(pB.d2 < c.z);
       if (__any_sync(kFull, undA || undB)) {  // rare: exact fp64 decision
-        if (undA) accA = opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
-        if (undB) accB = opening_accept64(W.pred[g + 1], T.x, T.y, T.z, T.th2);
+        const double ex = W.rec64 ? T.x64 : double(T.x), ey = W.rec64 ? T.y64 : double(T.y),
+                     ez = W.rec64 ? T.z64 : double(T.z);
+        if (undA) accA = opening_accept64(W.pred[g], ex, ey, ez, T.th2);
+        if (undB) accB = opening_accept64(W.pred[g + 1], ex, ey, ez, T.th2);
       }
       const uint32_t rejB = __ballot_sync(kFull, in && hasB && !accB);
       const uint32_t rejA = __ballot_sync(kFull, in && !accA);
@@ -268,24 +311,36 @@ __device__ __forceinline__ void mask_walk(const Walk& W, const Target& T, uint32
       sp = q + int(pushA);
     }
     if (__any_sync(kFull, accA)) {
-      a.add(accA, pA.dx, pA.dy, pA.dz, pA.d2, rA.w, T.eps2);
-      if (kQuad && l > 0) quad_at(a, pA, T.eps2, W.qf, g, accA);
+      walk_add(a, accA, pA, rA, W, g, T);
+      if constexpr (kQuad) { if (l > 0) quad_at(a, pA, T.eps2, W.qf, g, accA); }
     }
     if (__any_sync(kFull, accB)) {
-      a.add(accB, pB.dx, pB.dy, pB.dz, pB.d2, rB.w, T.eps2);
-      if (kQuad && l > 0) quad_at(a, pB, T.eps2, W.qf, g + 1u, accB);
+      walk_add(a, accB, pB, rB, W, g + 1u, T);
+      if constexpr (kQuad) { if (l > 0) quad_at(a, pB, T.eps2, W.qf, g + 1u, accB); }
     }
     a.n += accA;
     a.n += accB;
   }
 }
 
+template <bool kF64 = false>
 __device__ __forceinline__ Target load_target(const ForceParams& P, int64_t k, bool active) {
   Target T;
-  const float4 me = active ? P.leaves[k] : make_float4(0.f, 0.f, 0.f, 0.f);
-  T.x = me.x;
-  T.y = me.y;
-  T.z = me.z;
+  if constexpr (kF64) {  // NEXT-2: exact fp64 target, fp32 rounding for the filters
+    const double4 me = active ? P.leaves64[k] : make_double4(0.0, 0.0, 0.0, 0.0);
+    T.x64 = me.x;
+    T.y64 = me.y;
+    T.z64 = me.z;
+    T.x = float(me.x);
+    T.y = float(me.y);
+    T.z = float(me.z);
+    T.eps2_64 = P.eps2_64;
+  } else {
+    const float4 me = active ? P.leaves[k] : make_float4(0.f, 0.f, 0.f, 0.f);
+    T.x = me.x;
+    T.y = me.y;
+    T.z = me.z;
+  }
   T.th2 = P.th2;
   T.eps2 = P.eps2;
   return T;
@@ -303,10 +358,14 @@ __device__ __forceinline__ void owned_range(const ForceParams& P, int64_t& tb, i
 }
 
 // k: this lane's slot; k0: the warp's first slot (a multiple of 32 from 0).
+template <class AccT>
 __device__ __forceinline__ void store_result(const ForceParams& P, int64_t tb, int64_t k, int64_t k0, bool active,
-                                             const Acc& a, int lane) {
+                                             const AccT& a, int lane) {
   if (active) {
-    P.acc[k - tb] = make_float4(a.x, a.y, a.z, 0.f);
+    if constexpr (sizeof(a.x) == 8)
+      P.acc64[k - tb] = make_double4(a.x, a.y, a.z, 0.0);
+    else
+      P.acc[k - tb] = make_float4(a.x, a.y, a.z, 0.f);
     P.count[k - tb] = a.n;
   }
   const uint32_t tot = __reduce_add_sync(kFull, active ? a.n : 0u);
@@ -384,12 +443,16 @@ struct alignas(16) TgtPair {
   float2 px, py, pz, q;
 };
 
-template <bool kQuad>
+template <bool kQuad, bool kF64_ = false>
 struct alignas(16) V0Smem {
+  static constexpr bool kF64 = kF64_;
   TgtPair tgt[16];          // the warp's targets for the transposed test (paired)
-  float4 tpos[32];          // the warp's target positions (fp64 fallback)
-  RecPair frec[kCapF / 2];  // monopole / body records, all lanes
-  RecPair prec[kCapP / 2];  // monopole / body records, ...
+  float4 tpos[kF64 ? 1 : 32];   // the warp's target positions (fp64 fallback)
+  double4 tpos64[kF64 ? 32 : 1];  // NEXT-2 FP64 mode: exact target positions
+  RecPair frec[kF64 ? 1 : kCapF / 2];  // monopole / body records, all lanes
+  RecPair prec[kF64 ? 1 : kCapP / 2];  // monopole / body records, ...
+  double4 frec64[kF64 ? kCapF : 1];    // NEXT-2 FP64 mode: the same lists in fp64
+  double4 prec64[kF64 ? kCapP : 1];
   uint32_t pmsk[kCapP];     // ... for the lanes in the mask
   uint32_t astk[kCapA];
   uint2 tstk[kCapT];     // (id, mask of the targets that reached it)
@@ -543,11 +606,42 @@ __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Targe
   }
 }
 
-template <bool kSoft, bool kQuad>
-__global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(const ForceParams P) {
-  __shared__ V0Smem<kQuad> s_all[kV0Warps];
+// NEXT-2 FP64 mode dense phase: fp64 records, fp64 arithmetic.
+template <bool kSoft>
+__device__ __forceinline__ void dense_full64(V0Smem<false, true>& S, int nf, const Target& T, AccD& a) {
+#pragma unroll 2
+  for (int e = 0; e < nf; ++e) {
+    const double4 s = S.frec64[e];
+    interact64<kSoft>(a, s, s.w, T);
+  }
+  a.n += uint32_t(nf);
+}
+
+template <bool kSoft>
+__device__ __forceinline__ void dense_part64(V0Smem<false, true>& S, int np, const Target& T, AccD& a, int lane) {
+  uint32_t cnt = 0;
+#pragma unroll 2
+  for (int e = 0; e < np; ++e) {
+    const double4 s = S.prec64[e];
+    const bool on = (S.pmsk[e] >> lane) & 1u;
+    interact64<kSoft>(a, s, on ? s.w : 0.0, T);
+    cnt += on;
+  }
+  a.n += cnt;
+}
+
+#ifndef NBODY_V0_MINB_F64
+#define NBODY_V0_MINB_F64 4
+#endif
+
+template <bool kSoft, bool kQuad, bool kF64>
+__global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_MINB) void k_force_grouped(
+    const ForceParams P) {
+  static_assert(!(kQuad && kF64), "FP64 mode is monopole only");
+  using AccT = typename std::conditional<kF64, AccD, Acc>::type;
+  __shared__ V0Smem<kQuad, kF64> s_all[kV0Warps];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  V0Smem<kQuad>& S = s_all[w];
+  V0Smem<kQuad, kF64>& S = s_all[w];
   const float4* qf = kQuad ? in_reg(P.t.qf) : nullptr;
 #ifndef NBODY_GROUP
 #define NBODY_GROUP 32
@@ -560,8 +654,8 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   const bool active = k < te && lane < NBODY_GROUP;
   const uint32_t amask = __ballot_sync(kFull, active);
   if (amask == 0) return;
-  const Target T = load_target(P, k, active);
-  Acc a;
+  const Target T = load_target<kF64>(P, k, active);
+  AccT a;
   const uint32_t lt = (1u << lane) - 1u;
   const Walk W = make_walk(P);
   const float4* tfp = in_reg(P.t.tf);
@@ -580,14 +674,20 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   const float gx = 0.5f * blx + 0.5f * bhx, gy = 0.5f * bly + 0.5f * bhy, gz = 0.5f * blz + 0.5f * bhz;
   float kk1, kk0;
   {
-    const float ux = active ? T.x - gx : 0.f, uy = active ? T.y - gy : 0.f, uz = active ? T.z - gz : 0.f;
+    // x' = fl32(x - g) (FP64 mode: of the exact fp64 difference)
+    const float ux = !active ? 0.f : kF64 ? float(T.x64 - double(gx)) : T.x - gx;
+    const float uy = !active ? 0.f : kF64 ? float(T.y64 - double(gy)) : T.y - gy;
+    const float uz = !active ? 0.f : kF64 ? float(T.z64 - double(gz)) : T.z - gz;
     const double u2 = fma(double(uz), double(uz), fma(double(uy), double(uy), double(ux) * double(ux)));
     TgtPair& tp = S.tgt[lane >> 1];
     reinterpret_cast<float*>(&tp.px)[lane & 1] = 2.f * ux;
     reinterpret_cast<float*>(&tp.py)[lane & 1] = 2.f * uy;
     reinterpret_cast<float*>(&tp.pz)[lane & 1] = 2.f * uz;
     reinterpret_cast<float*>(&tp.q)[lane & 1] = float(-u2);
-    S.tpos[lane] = make_float4(T.x, T.y, T.z, 0.f);
+    if constexpr (kF64)
+      S.tpos64[lane] = make_double4(T.x64, T.y64, T.z64, 0.0);
+    else
+      S.tpos[lane] = make_float4(T.x, T.y, T.z, 0.f);
     // b >= |x - g| = |x'| (1 + O(u)): 4e-7 > 2u + rounding of the bound
     const float b = __fmul_ru(warp_maxf(__fsqrt_ru(__double2float_ru(u2))), 1.f + 4e-7f);
     const float R = P.grid->R;
@@ -607,19 +707,26 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   // Append (record r, lane mask msk) to the dense lists: full when every
   // active lane interacts with it.
   // active lane interacts with it.  id: the node (quadrupole source), 0 for a body.
-  auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id) {
+  // g: the node id (FP64 mode reads its fp64 record rec64[g]).
+  auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id, uint32_t g) {
     const bool full = want && msk == amask;
     const bool part = want && msk != amask;
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
     if (full) {
       const int pos = nf + __popc(bf & lt);
-      S.frec[pos >> 1].put(pos & 1, r);
+      if constexpr (kF64)
+        S.frec64[pos] = P.t.rec64[g];
+      else
+        S.frec[pos >> 1].put(pos & 1, r);
       if (kQuad) S.fid[pos] = id;
     }
     if (part) {
       const int pos = np + __popc(bp & lt);
-      S.prec[pos >> 1].put(pos & 1, r);
+      if constexpr (kF64)
+        S.prec64[pos] = P.t.rec64[g];
+      else
+        S.prec[pos >> 1].put(pos & 1, r);
       S.pmsk[pos] = msk;
       if (kQuad) S.pid[pos] = id;
     }
@@ -656,13 +763,19 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
   auto flush = [&](bool all) {
     __syncwarp();
     if (nf > kCapF - 32 || (all && nf > 0)) {
-      dense_full<kSoft, kQuad>(S, nf, T, a, qf, lane);
+      if constexpr (kF64)
+        dense_full64<kSoft>(S, nf, T, a);
+      else
+        dense_full<kSoft, kQuad>(S, nf, T, a, qf, lane);
       K6STAT(10, 1);
       K6STAT(11, (nf + 1) >> 1);
       nf = 0;
     }
     if (np > kCapP - 32 || (all && np > 0)) {
-      dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
+      if constexpr (kF64)
+        dense_part64<kSoft>(S, np, T, a, lane);
+      else
+        dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
       K6STAT(12, 1);
       K6STAT(13, (np + 1) >> 1);
 #ifdef NBODY_K6_STATS
@@ -743,14 +856,21 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
           const double4 pd = W.pred[g];
           do {
             const int t = __ffs(int(und)) - 1;
-            const float4 tp = S.tpos[t];
-            if (opening_accept64(pd, tp.x, tp.y, tp.z, T.th2)) am |= 1u << t; else rm |= 1u << t;
+            bool acc;
+            if constexpr (kF64) {
+              const double4 tp = S.tpos64[t];
+              acc = opening_accept64(pd, tp.x, tp.y, tp.z, T.th2);
+            } else {
+              const float4 tp = S.tpos[t];
+              acc = opening_accept64(pd, tp.x, tp.y, tp.z, T.th2);
+            }
+            if (acc) am |= 1u << t; else rm |= 1u << t;
             und &= und - 1u;
           } while (und);
         }
       }
       if (g >= leaf0 && g - kid0 < 32u) am &= ~(1u << (g - kid0));  // a leaf never acts on itself
-      append(am != 0u, r, am, g < leaf0 ? g : 0u);
+      append(am != 0u, r, am, g < leaf0 ? g : 0u, g);
       // children of opened nodes, with the mask of the targets that opened them
       const int l = L - 31 + __clz(int(g));
       const bool two = rm && (((2u * g + 1u) << (l - 1)) - leaf0) < n;
@@ -826,7 +946,7 @@ __global__ __launch_bounds__(32 * kV0Warps, NBODY_V0_MINB) void k_force_grouped(
       }
       uint32_t msk = amask;
       if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
-      append(cls == 1, r, msk, g < leaf0 ? g : 0u);
+      append(cls == 1, r, msk, g < leaf0 ? g : 0u, g);
       const uint32_t bt = __ballot_sync(kFull, cls == 3);
       if (cls == 3) S.tstk[nt + __popc(bt & lt)] = make_uint2(g, amask);
       nt += __popc(bt);
@@ -866,15 +986,20 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
       k_force_maskstack<false><<<grid, 32 * kV1Warps, 0, s>>>(p);
   } else {
     const unsigned grid = unsigned(((nt + NBODY_GROUP - 1) / NBODY_GROUP + kV0Warps - 1) / kV0Warps);
-    const bool soft = p.eps2 > 0.f;
-    if (soft && !quad)
-      k_force_grouped<true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    const bool soft = p.t.rec64 ? p.eps2_64 > 0.0 : p.eps2 > 0.f;
+    if (p.t.rec64) {  // NEXT-2 FP64 mode (monopole, variant 0)
+      if (soft)
+        k_force_grouped<true, false, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+      else
+        k_force_grouped<false, false, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+    } else if (soft && !quad)
+      k_force_grouped<true, false, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
     else if (!soft && !quad)
-      k_force_grouped<false, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
+      k_force_grouped<false, false, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
     else if (soft)
-      k_force_grouped<true, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+      k_force_grouped<true, true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
     else
-      k_force_grouped<false, true><<<grid, 32 * kV0Warps, 0, s>>>(p);
+      k_force_grouped<false, true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
   }
 }
 

@@ -61,6 +61,64 @@ __global__ __launch_bounds__(256) void k_scatter1(const uint32_t* __restrict__ s
   out[__float_as_int(vi[i].w)] = src[i];
 }
 
+// ---- NEXT-2 FP64 mode: the same helpers on fp64 bodies -------------------
+// Leapfrog in fp64 (the oracle's O8 on fp64 state: v + a dt, x + v dt).
+__global__ __launch_bounds__(256) void k_leapfrog_f64(const double4* __restrict__ pm_in,
+                                                      const double4* __restrict__ vi_in,
+                                                      const double4* __restrict__ acc, int64_t n, double dt,
+                                                      double4* __restrict__ pm_out, double4* __restrict__ vi_out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double4 p = pm_in[i], v = vi_in[i];
+  const double4 a = acc[i];
+  v.x = __dadd_rn(v.x, __dmul_rn(a.x, dt));
+  v.y = __dadd_rn(v.y, __dmul_rn(a.y, dt));
+  v.z = __dadd_rn(v.z, __dmul_rn(a.z, dt));
+  p.x = __dadd_rn(p.x, __dmul_rn(v.x, dt));
+  p.y = __dadd_rn(p.y, __dmul_rn(v.y, dt));
+  p.z = __dadd_rn(p.z, __dmul_rn(v.z, dt));
+  pm_out[i] = p;
+  vi_out[i] = v;
+}
+
+__global__ __launch_bounds__(256) void k_pack_f64(const double* __restrict__ pos, const double* __restrict__ vel,
+                                                  const double* __restrict__ mass, int64_t n,
+                                                  double4* __restrict__ pm, double4* __restrict__ vi,
+                                                  int* __restrict__ bad) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const double x = pos[3 * i], y = pos[3 * i + 1], z = pos[3 * i + 2];
+  const double u = vel[3 * i], v = vel[3 * i + 1], w = vel[3 * i + 2];
+  const double m = mass[i];
+  int flag = 0;
+  if (!(isfinite(x) && isfinite(y) && isfinite(z) && isfinite(u) && isfinite(v) && isfinite(w))) flag |= 1;
+  if (!(isfinite(m) && m > 0.0)) flag |= 2;
+  if (flag) atomicOr(bad, flag);
+  pm[i] = make_double4(x, y, z, m);
+  vi[i] = make_double4(u, v, w, double(i));
+}
+
+template <class Out>
+__global__ __launch_bounds__(256) void k_scatter3_f64(const double4* __restrict__ src,
+                                                      const double4* __restrict__ vi, int64_t n,
+                                                      Out* __restrict__ out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int64_t id = int64_t(vi[i].w);
+  const double4 s = src[i];
+  out[3 * id] = Out(s.x);
+  out[3 * id + 1] = Out(s.y);
+  out[3 * id + 2] = Out(s.z);
+}
+
+__global__ __launch_bounds__(256) void k_scatter1_f64(const uint32_t* __restrict__ src,
+                                                      const double4* __restrict__ vi, int64_t n,
+                                                      uint32_t* __restrict__ out) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  out[int64_t(vi[i].w)] = src[i];
+}
+
 __global__ __launch_bounds__(256) void k_fill2(float2* __restrict__ p, int64_t count, float2 v) {
   const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   if (i < count) p[i] = v;
@@ -92,6 +150,32 @@ void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s) {
   if (n <= 0) return;
   k_scatter1<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
+}
+
+void launch_leapfrog_f64(const double4* pm_in, const double4* vi_in, const double4* acc, int64_t n, double dt,
+                         double4* pm_out, double4* vi_out, cudaStream_t s) {
+  if (n <= 0) return;
+  k_leapfrog_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, n, dt, pm_out, vi_out);
+}
+
+void launch_pack_bodies_f64(const double* pos, const double* vel, const double* mass, int64_t n, double4* pm,
+                            double4* vi, int* bad, cudaStream_t s) {
+  k_pack_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(pos, vel, mass, n, pm, vi, bad);
+}
+
+void launch_scatter_by_id3_f64(const double4* src, const double4* vi, int64_t n, double* out, cudaStream_t s) {
+  if (n <= 0) return;
+  k_scatter3_f64<double><<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
+}
+
+void launch_scatter_by_id3_f64to32(const double4* src, const double4* vi, int64_t n, float* out, cudaStream_t s) {
+  if (n <= 0) return;
+  k_scatter3_f64<float><<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
+}
+
+void launch_scatter_by_id1_f64(const uint32_t* src, const double4* vi, int64_t n, uint32_t* out, cudaStream_t s) {
+  if (n <= 0) return;
+  k_scatter1_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
 }
 
 }  // namespace nb

@@ -28,6 +28,20 @@ def _ptr(a) -> int:
     raise TypeError(f"unsupported buffer type {type(a)}")
 
 
+def _f64(a, n, cols):
+    if isinstance(a, np.ndarray):
+        a = np.ascontiguousarray(a, dtype=np.float64)
+        if a.size != n * cols:
+            raise ValueError(f"expected {n}x{cols} values, got {a.shape}")
+        return a
+    if hasattr(a, "data_ptr"):
+        import torch
+        if a.dtype != torch.float64 or a.numel() != n * cols:
+            raise ValueError("expected a float64 tensor of n*cols elements")
+        return a.contiguous()
+    raise TypeError(type(a))
+
+
 def _f32(a, n, cols):
     if isinstance(a, np.ndarray):
         a = np.ascontiguousarray(a, dtype=np.float32)
@@ -47,7 +61,7 @@ class NBody:
 
     def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
                  stream=None, use_graph: bool = True, traversal: int = 0, device=None, multipole: int = 1,
-                 balance: bool = False):
+                 balance: bool = False, precision: int = 32):
         self.lib = _capi.load()
         self.n = int(n)
         if device is None:  # follow PyTorch's current device when torch has one
@@ -73,6 +87,9 @@ class NBody:
             self.set_option(_capi.NBODY_OPT_MULTIPOLE, multipole)
         if balance:  # NEXT-3(i) cost-weighted ranges (peer exchange only)
             self.set_option(_capi.NBODY_OPT_BALANCE, 1)
+        self.precision = int(precision)
+        if self.precision != 32:  # NEXT-2 FP64 mode
+            self.set_option(_capi.NBODY_OPT_PRECISION, self.precision)
         if stream is not None:
             self.set_option(_capi.NBODY_OPT_STREAM, int(stream))
 
@@ -102,6 +119,10 @@ class NBody:
         self._ck(self.lib.nbody_set_option(self.h, int(opt), int(value)))
 
     def set_bodies(self, pos, vel, mass):
+        if self.precision == 64:
+            p, v, m = _f64(pos, self.n, 3), _f64(vel, self.n, 3), _f64(mass, self.n, 1)
+            self._ck(self.lib.nbody_set_bodies64(self.h, _ptr(p), _ptr(v), _ptr(m)))
+            return
         p, v, m = _f32(pos, self.n, 3), _f32(vel, self.n, 3), _f32(mass, self.n, 1)
         self._ck(self.lib.nbody_set_bodies(self.h, _ptr(p), _ptr(v), _ptr(m)))
 
@@ -127,6 +148,35 @@ class NBody:
 
     def get_velocities(self, out=None):
         return self._get3(self.lib.nbody_get_velocities, out)
+
+    # NEXT-2 FP64 mode getters
+    def _get3d(self, fn, out=None):
+        out = np.empty((self.n, 3), np.float64) if out is None else out
+        self._ck(fn(self.h, _ptr(out)))
+        return out
+
+    def get_accel64(self, out=None):
+        return self._get3d(self.lib.nbody_get_accel64, out)
+
+    def get_positions64(self, out=None):
+        return self._get3d(self.lib.nbody_get_positions64, out)
+
+    def get_velocities64(self, out=None):
+        return self._get3d(self.lib.nbody_get_velocities64, out)
+
+    def get_state64(self):
+        pm = np.empty((self.n, 4), np.float64)
+        vi = np.empty((self.n, 4), np.float64)
+        self._ck(self.lib.nbody_get_state64(self.h, _ptr(pm), _ptr(vi)))
+        return pm, vi
+
+    def debug_level64(self, level: int):
+        cnt = C.c_int64()
+        self._ck(self.lib.nbody_debug_level64(self.h, int(level), C.byref(cnt), None, None))
+        rec = np.empty((cnt.value, 4), np.float64)
+        box = np.empty((cnt.value, 6), np.float64)
+        self._ck(self.lib.nbody_debug_level64(self.h, int(level), C.byref(cnt), _ptr(rec), _ptr(box)))
+        return rec, box
 
     def get_interactions(self, out=None):
         out = np.empty(self.n, np.uint32) if out is None else out
@@ -232,6 +282,7 @@ class NBody:
         c = cnt.value
         pred = np.empty((c, 4), np.float64)
         rec = np.empty((c, 4), np.float32)
-        box = np.empty((c, 6), np.float32)
-        self._ck(self.lib.nbody_debug_level(self.h, int(level), C.byref(cnt), _ptr(pred), _ptr(rec), _ptr(box)))
+        box = np.empty((c, 6), np.float32) if self.precision == 32 else None  # fp64: debug_level64
+        self._ck(self.lib.nbody_debug_level(self.h, int(level), C.byref(cnt), _ptr(pred), _ptr(rec),
+                                            _ptr(box) if box is not None else None))
         return pred, rec, box
