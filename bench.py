@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--balance", choices=["cost", "equal"], default="cost",
                     help="multi-GPU ranges (peer exchange): cost-weighted from the last pass (NEXT-3(i), default) "
                          "or equal slices [A21]")
+    ap.add_argument("--precision", type=int, choices=[32, 64], default=32,
+                    help="32: fp32 state and interactions (default); 64: the paper's FP64 throughout (NEXT-2)")
     ap.add_argument("--sort-every", type=int, default=1,
                     help="ablation: tree reuse, re-sort every k-th step (NEXT-3(iii)); 1 = Alg. 6")
     return ap.parse_args()
@@ -157,8 +159,9 @@ def cpu_oracle_sample(pos, vel, mass, cfg, target_seconds, seed=0):
     rng = np.random.default_rng(seed)
     probe = np.sort(rng.choice(n, min(n, 500), replace=False))
     t0 = time.perf_counter()
+    prec = 64 if pos.dtype == np.float64 else 32
     r = O.step(pos, vel, mass, theta=cfg["theta"], eps=cfg["eps"], dt=cfg["dt"], key_bits=16, integrate=False,
-               targets=probe)
+               targets=probe, precision=prec)
     t_all = time.perf_counter() - t0
     tf0 = time.perf_counter()
     r.tree.force(cfg["theta"], cfg["eps"], probe)
@@ -218,9 +221,12 @@ def run_ours(args, cfg, world, rank, local):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     n = cfg["n"]
-    pos, vel, mass = generate(cfg["workload"], n, cfg["seed"])
+    f64 = args.precision == 64
+    pos, vel, mass = generate(cfg["workload"], n, cfg["seed"], np.float64 if f64 else np.float32)
     stream = torch.cuda.Stream()
-    sim = NBody(n, cfg["theta"], cfg["eps"], cfg["dt"], key_bits=16, stream=stream.cuda_stream)
+    sim = NBody(n, cfg["theta"], cfg["eps"], cfg["dt"], key_bits=16, stream=stream.cuda_stream,
+                precision=args.precision)
+    cfg["precision"] = args.precision
     if args.sort_every != 1:
         sim.set_option(7, args.sort_every)  # NBODY_OPT_SORT_EVERY
         cfg["sort_every"] = args.sort_every
@@ -285,13 +291,15 @@ def run_ours(args, cfg, world, rank, local):
     peaks = measured_peaks()
     nsm = torch.cuda.get_device_properties(local).multi_processor_count
     fmax = float(peaks.get("sm_max_mhz", 1965.0))
-    peak_tflops = 2 * 128 * nsm * fmax * 1e6 / 1e12  # FP32 FFMA lanes x 2 flop x SMs x max clock
+    lanes = 64 if f64 else 128  # FP64: 64 DFMA lanes/SM (measured 59/clk, scripts/micro/pipe_rates.cu)
+    peak_tflops = 2 * lanes * nsm * fmax * 1e6 / 1e12  # FMA lanes x 2 flop x SMs x max clock
     achieved = force_flops / (force_ms / 1e3) / 1e12
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak_tflops, "unit": "TFLOP/s",
-                "frac": achieved / peak_tflops, "traffic": ncu_traffic(),
+                "frac": achieved / peak_tflops, "traffic": None if f64 else ncu_traffic(),
                 "kernel": "k_force (CALCULATEFORCE)", "flops_per_interaction": FLOPS_PER_INTERACTION,
                 "kernel_ms": force_ms,
-                "peak_basis": f"FP32 pipe 2 flop x 128 lanes x {nsm} SMs x {fmax:.0f} MHz (sm_max, MEASURED_PEAKS.json)",
+                "peak_basis": f"{'FP64' if f64 else 'FP32'} pipe 2 flop x {lanes} lanes x {nsm} SMs x {fmax:.0f} MHz "
+                              "(sm_max, MEASURED_PEAKS.json)",
                 "share_of_step": force_ms / ms}
 
     # End to end through the public API: pinned host inputs -> step -> host result.
@@ -300,25 +308,27 @@ def run_ours(args, cfg, world, rank, local):
         hp = torch.from_numpy(pos).pin_memory()
         hv = torch.from_numpy(vel).pin_memory()
         hm = torch.from_numpy(mass).pin_memory()
-        out = torch.empty((n, 3), dtype=torch.float32).pin_memory()
+        out = torch.empty((n, 3), dtype=torch.float64 if f64 else torch.float32).pin_memory()
+        get_pos = sim.get_positions64 if f64 else sim.get_positions
         # every rank loads the full input and reads the full result (the state
         # is replicated after each step's all-gather)
         sim.set_bodies(hp, hv, hm)
         sim.step(1)
-        sim.get_positions(out)
+        get_pos(out)
         barrier()
         t0 = time.perf_counter()
         for _ in range(args.steps):
             sim.set_bodies(hp, hv, hm)
             sim.step(1)
-            sim.get_positions(out)
+            get_pos(out)
         barrier()
         e2e_ms = 1e3 * (time.perf_counter() - t0) / args.steps
         if world > 1:
             from paper_conf_sc_casselldahg24_b200.dist import max_over_ranks
             e2e_ms = max_over_ranks(e2e_ms, device="cuda")
-        e2e = {"value": n / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": 28 * n * world,
-               "d2h_bytes_per_step": 12 * n * world, "ms_per_step": e2e_ms,
+        w = 2 if f64 else 1
+        e2e = {"value": n / (e2e_ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": 28 * w * n * world,
+               "d2h_bytes_per_step": 12 * w * n * world, "ms_per_step": e2e_ms,
                "path": "nbody_set_bodies(pinned host) + nbody_step(1) + nbody_get_positions(pinned host), per rank"}
 
     cpu = None
@@ -330,7 +340,8 @@ def run_ours(args, cfg, world, rank, local):
     if rank == 0:
         line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
-                "vs_baseline": None, "dtype": "f32 (fp64 tree moments, key grid and opening test)",
+                "vs_baseline": None,
+                "dtype": "f64" if f64 else "f32 (fp64 tree moments, key grid and opening test)",
                 "data": "synthetic", "impl": "ours",
                 "config": config_json(cfg, world),
                 "interactions_per_s": inter / (ms / 1e3), "interactions_per_body": inter / n,

@@ -10,8 +10,9 @@ template <int OP>
 __global__ void k(float* out, float a0, float b0, long long* cyc) {
   float2 x[8], y = make_float2(a0, b0), z = make_float2(b0, a0);
   float s[8];
+  double d[8], dy = a0, dz = b0;
 #pragma unroll
-  for (int i = 0; i < 8; ++i) { x[i] = make_float2(a0 + i, b0 - i); s[i] = a0 * i; }
+  for (int i = 0; i < 8; ++i) { x[i] = make_float2(a0 + i, b0 - i); s[i] = a0 * i; d[i] = b0 * i; }
   __syncthreads();
   long long t0 = clock64();
   for (int it = 0; it < kIters; ++it) {
@@ -25,12 +26,13 @@ __global__ void k(float* out, float a0, float b0, long long* cyc) {
       if (OP == 5) { float r; asm volatile("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(s[i])); s[i] = r; }
       if (OP == 6) { s[i] = fmaf(s[i], y.x, z.x); x[i] = __ffma2_rn(x[i], y, z); }  // mix
       if (OP == 7) { x[i] = __ffma2_rn(x[i], x[i], z); }  // FFMA2 with a repeated operand
+      if (OP == 8) { d[i] = fma(d[i], dy, dz); }           // DFMA
     }
   }
   long long t1 = clock64();
   float acc = 0.f;
 #pragma unroll
-  for (int i = 0; i < 8; ++i) acc += x[i].x + x[i].y + s[i];
+  for (int i = 0; i < 8; ++i) acc += x[i].x + x[i].y + s[i] + float(d[i]);
   out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
   if (threadIdx.x == 0 && blockIdx.x == 0) *cyc = t1 - t0;
 }
@@ -75,6 +77,7 @@ int main() {
     run<7>("FFMA2 repeated operand", sms, thr);
     run<5>("MUFU.RSQ", sms, thr);
     run<6>("FFMA + FFMA2 mix (2 inst)", sms, thr);
+    run<8>("DFMA", sms, thr);
   }
   return 0;
 }
