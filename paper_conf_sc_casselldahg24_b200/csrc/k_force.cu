@@ -417,6 +417,9 @@ constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 #ifndef NBODY_CAP_P
 #define NBODY_CAP_P 64
 #endif
+#ifndef NBODY_LEAF_DIRECT
+#define NBODY_LEAF_DIRECT 1
+#endif
 constexpr int kCapF = NBODY_CAP_F;  // dense list: entries every active lane interacts with
 constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 
@@ -874,8 +877,29 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       // children of opened nodes, with the mask of the targets that opened them
       const int l = L - 31 + __clz(int(g));
       const bool two = rm && (((2u * g + 1u) << (l - 1)) - leaf0) < n;
+#if NBODY_LEAF_DIRECT
+      // Children that are leaves are accepted by every target that reaches
+      // them (except a target by itself), so they go straight to the dense
+      // lists with the opening mask instead of through another T slot.
+      const bool lv = rm != 0u && l == 1;
+      if (__any_sync(kFull, lv)) {
+        float4 ra = make_float4(0.f, 0.f, 0.f, 0.f), rb = ra;
+        if (lv && !kF64) load_pair(W.rec + 2u * g, ra, rb);  // ids < 2^(L+1): in bounds
+        const uint32_t ca = 2u * g, cb = ca + 1u;
+        uint32_t ma = lv ? rm : 0u, mb = lv && two ? rm : 0u;
+        if (ca - kid0 < 32u) ma &= ~(1u << (ca - kid0));
+        if (cb - kid0 < 32u) mb &= ~(1u << (cb - kid0));
+        flush(false);
+        append(ma != 0u, ra, ma, 0u, ca);
+        flush(false);
+        append(mb != 0u, rb, mb, 0u, cb);
+      }
+      const bool push = rm != 0u && nt + 64 <= kCapT && !lv;
+      const bool room = nt + 64 <= kCapT || lv;
+#else
       const bool room = nt + 64 <= kCapT;
       const bool push = rm != 0u && room;
+#endif
       const uint32_t b1 = __ballot_sync(kFull, push);
       const uint32_t b2 = __ballot_sync(kFull, push && two);
       if (push) {
