@@ -156,6 +156,24 @@ nbody_status nbody_set_bodies(nbody_ctx *ctx, const float *pos, const float *vel
  * NBODY_EINVAL in mode 32, for null pointers or invalid values [A18]. */
 nbody_status nbody_set_bodies64(nbody_ctx *ctx, const double *pos, const double *vel, const double *mass);
 
+/* Pipelined host transfers (fp32 mode).  nbody_set_bodies_async does what
+ * nbody_set_bodies does, but the copy of pos[n][3], vel[n][3], mass[n]
+ * runs on the context's host->device copy stream into one of two device
+ * staging buffers, and the packing runs on the context stream after it, so
+ * the copy overlaps the steps still queued there.  nbody_get_positions_async
+ * enqueues the by-id gather of the current positions on the context
+ * stream and the copy into out[n][3] on the device->host copy stream
+ * (double-buffered), so the copy overlaps the next steps.  Both return
+ * without waiting: the caller keeps the input buffers unchanged and does
+ * not read `out` until nbody_sync; host buffers should be pinned for the
+ * copies to overlap.  Input validation [A18] is deferred: nbody_sync
+ * returns NBODY_EINVAL if any input set since the last sync was invalid
+ * (the steps computed from it are then meaningless).  The staging buffers
+ * (80 B per body) are allocated on first use.  NBODY_EINVAL in FP64 mode or
+ * for null pointers. */
+nbody_status nbody_set_bodies_async(nbody_ctx *ctx, const float *pos, const float *vel, const float *mass);
+nbody_status nbody_get_positions_async(nbody_ctx *ctx, float *out);
+
 /* Stages 1-5 of Alg. 6 at the current positions (no UPDATEPOSITION):
  * bbox, keys, sort, permute, build, force.  Afterwards slot order is the
  * new Hilbert order and nbody_get_accel returns a(x_t).  Asynchronous. */
@@ -165,7 +183,8 @@ nbody_status nbody_compute_accel(nbody_ctx *ctx);
  * v += a dt, x += v dt [A14]).  Asynchronous on the context stream. */
 nbody_status nbody_step(nbody_ctx *ctx, int nsteps);
 
-/* Wait for all work issued on the context stream. */
+/* Wait for all work issued on the context stream and the copy streams;
+ * reports a deferred input error of nbody_set_bodies_async. */
 nbody_status nbody_sync(nbody_ctx *ctx);
 
 /* a(x) of the last force pass, out[n][3] by id (fp32). */

@@ -58,6 +58,8 @@ SIGNATURES = {
     "nbody_create": (_S, [_I64, C.c_double, C.c_double, C.c_double, C.POINTER(_P)]),
     "nbody_set_option": (_S, [_P, C.c_int, _I64]),
     "nbody_set_bodies": (_S, [_P, _P, _P, _P]),
+    "nbody_set_bodies_async": (_S, [_P, _P, _P, _P]),
+    "nbody_get_positions_async": (_S, [_P, _P]),
     "nbody_compute_accel": (_S, [_P]),
     "nbody_step": (_S, [_P, C.c_int]),
     "nbody_sync": (_S, [_P]),

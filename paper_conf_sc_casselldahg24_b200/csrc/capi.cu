@@ -105,6 +105,14 @@ struct nbody_ctx {
   uint32_t* gcost = nullptr;        // [ceil(n/32)] interactions per 32-slot group, last pass
   int64_t* dpart = nullptr;         // [kMaxPeers + 1] slot boundaries of the next pass
   int64_t* dpart_used = nullptr;    // [kMaxPeers + 1] boundaries of the last pass
+  // pipelined host transfers (nbody_set_bodies_async / nbody_get_positions_async)
+  cudaStream_t cstream = nullptr;   // copy stream, host -> device
+  cudaStream_t ostream = nullptr;   // copy stream, device -> host (separate: it waits for steps)
+  char* xfer = nullptr;             // in_stage[2] (28 B/body) + out_stage[2] (12 B/body)
+  int* bad_async = nullptr;         // validation flags of async input sets since the last sync
+  cudaEvent_t ev_in_copied[2] = {}, ev_in_used[2] = {}, ev_out_ready[2] = {}, ev_out_copied[2] = {};
+  bool ev_in_used_rec[2] = {}, ev_out_copied_rec[2] = {};
+  int slot_in = 0, slot_out = 0;
 };
 
 namespace {
@@ -776,6 +784,82 @@ nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, 
   return NBODY_OK;
 }
 
+// Lazily create the copy stream, events and staging buffers of the
+// pipelined transfers.
+static nbody_status ensure_xfer(nbody_ctx* c) {
+  if (c->xfer) return NBODY_OK;
+  const size_t n = size_t(c->n);
+  CK(cudaStreamCreateWithFlags(&c->cstream, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&c->ostream, cudaStreamNonBlocking));
+  for (int k = 0; k < 2; ++k) {
+    CK(cudaEventCreateWithFlags(&c->ev_in_copied[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_in_used[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_out_ready[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->ev_out_copied[k], cudaEventDisableTiming));
+  }
+  void* p = nullptr;
+  const cudaError_t e = cudaMalloc(&p, align_up(2 * 28 * n) + align_up(2 * 12 * n) + 256);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(c, NBODY_ENOMEM, "staging buffers of the pipelined transfers");
+  }
+  c->xfer = static_cast<char*>(p);
+  c->bad_async = reinterpret_cast<int*>(c->xfer + align_up(2 * 28 * n) + align_up(2 * 12 * n));
+  CK(cudaMemsetAsync(c->bad_async, 0, sizeof(int), c->stream));
+  return NBODY_OK;
+}
+
+nbody_status nbody_set_bodies_async(nbody_ctx* c, const float* pos, const float* vel, const float* mass) {
+  CHECK_CTX(c);
+  if (c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: use nbody_set_bodies64");
+  if (!pos || !vel || !mass) return fail(c, NBODY_EINVAL, "null input");
+  nbody_status st = ensure_xfer(c);
+  if (st != NBODY_OK) return st;
+  const size_t n = size_t(c->n);
+  const int k = c->slot_in;
+  c->slot_in ^= 1;
+  float* in = reinterpret_cast<float*>(c->xfer + k * 28 * n);
+  // the staging buffer is free once the packing of the set before last ran
+  if (c->ev_in_used_rec[k]) CK(cudaStreamWaitEvent(c->cstream, c->ev_in_used[k], 0));
+  CK(cudaMemcpyAsync(in, pos, 12 * n, cudaMemcpyDefault, c->cstream));
+  CK(cudaMemcpyAsync(in + 3 * n, vel, 12 * n, cudaMemcpyDefault, c->cstream));
+  CK(cudaMemcpyAsync(in + 6 * n, mass, 4 * n, cudaMemcpyDefault, c->cstream));
+  CK(cudaEventRecord(c->ev_in_copied[k], c->cstream));
+  CK(cudaStreamWaitEvent(c->stream, c->ev_in_copied[k], 0));
+  launch_pack_bodies(in, in + 3 * n, in + 6 * n, c->n, c->pm[0], c->vi[0], c->bad_async, c->stream);
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(c->ev_in_used[k], c->stream));
+  c->ev_in_used_rec[k] = true;
+  c->loaded = true;
+  c->have_force = false;
+  c->keys_dbg_valid = false;
+  c->steps = 0;
+  return NBODY_OK;
+}
+
+nbody_status nbody_get_positions_async(nbody_ctx* c, float* out) {
+  CHECK_CTX(c);
+  if (c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: use nbody_get_positions64");
+  if (!out) return fail(c, NBODY_EINVAL, "null output");
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  nbody_status st = ensure_xfer(c);
+  if (st != NBODY_OK) return st;
+  const size_t n = size_t(c->n);
+  const int k = c->slot_out;
+  c->slot_out ^= 1;
+  float* stage = reinterpret_cast<float*>(c->xfer + align_up(2 * 28 * n) + k * 12 * n);
+  // the staging buffer is free once the copy-out issued two calls ago is done
+  if (c->ev_out_copied_rec[k]) CK(cudaStreamWaitEvent(c->stream, c->ev_out_copied[k], 0));
+  launch_scatter_by_id3(c->pm[0], c->vi[0], c->n, stage, c->stream);
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(c->ev_out_ready[k], c->stream));
+  CK(cudaStreamWaitEvent(c->ostream, c->ev_out_ready[k], 0));
+  CK(cudaMemcpyAsync(out, stage, 12 * n, cudaMemcpyDefault, c->ostream));
+  CK(cudaEventRecord(c->ev_out_copied[k], c->ostream));
+  c->ev_out_copied_rec[k] = true;
+  return NBODY_OK;
+}
+
 nbody_status nbody_compute_accel(nbody_ctx* c) {
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
@@ -817,7 +901,19 @@ nbody_status nbody_step(nbody_ctx* c, int nsteps) {
 
 nbody_status nbody_sync(nbody_ctx* c) {
   CHECK_CTX(c);
-  return sync_stream(c);
+  if (c->cstream) CK(cudaStreamSynchronize(c->cstream));
+  if (c->ostream) CK(cudaStreamSynchronize(c->ostream));
+  const nbody_status st = sync_stream(c);
+  if (st != NBODY_OK || !c->bad_async) return st;
+  int bad = 0;
+  CK(cudaMemcpy(&bad, c->bad_async, sizeof(int), cudaMemcpyDeviceToHost));
+  if (bad) {
+    CK(cudaMemset(c->bad_async, 0, sizeof(int)));
+    c->loaded = false;
+    return fail(c, NBODY_EINVAL, (bad & 2) ? "an async input set had masses that are not finite and > 0"
+                                           : "an async input set had a non-finite position or velocity");
+  }
+  return NBODY_OK;
 }
 
 // out[id][3] <- src[i].xyz for the slots [b, e) (src[i] belongs to slot b + i).
@@ -1343,6 +1439,15 @@ void nbody_destroy(nbody_ctx* c) {
   if (c->arena64) cudaFree(c->arena64);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
+  for (cudaStream_t cs : {c->cstream, c->ostream})
+    if (cs) {
+      cudaStreamSynchronize(cs);
+      cudaStreamDestroy(cs);
+    }
+  for (int k = 0; k < 2; ++k)
+    for (cudaEvent_t e : {c->ev_in_copied[k], c->ev_in_used[k], c->ev_out_ready[k], c->ev_out_copied[k]})
+      if (e) cudaEventDestroy(e);
+  if (c->xfer) cudaFree(c->xfer);
   if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
   if (c->own_stream) cudaStreamDestroy(c->own_stream);
   cudaGetLastError();

@@ -5,8 +5,8 @@
 // reduction order, so it is deterministic and bit-identical to any other
 // correct min/max.  K2 quantises in fp64 with explicitly rounded operations
 // (no contraction possible in the (x - lo) * inv form) [A9][A16][A17] and
-// encodes the cell with a branch-free form of Skilling's transpose plus a
-// magic-number bit interleave.  HBM bound: 16 B read per body (K1), 16 B read
+// encodes the cell with Skilling's transform as a 48-state table-driven
+// automaton (two levels per shared-memory lookup).  HBM bound: 16 B read per body (K1), 16 B read
 // + 4/8 B written per body (K2).
 #include <float.h>
 
@@ -159,42 +159,107 @@ __global__ void k_bbox_final_f64(const double* __restrict__ partial, int nparts,
   }
 }
 
-// Spread the low 21 bits of v so that bit q lands at bit 3q.
-__device__ __forceinline__ unsigned long long spread3(uint32_t v) {
-  unsigned long long x = v & 0x1fffffull;
-  x = (x | (x << 32)) & 0x001f00000000ffffull;
-  x = (x | (x << 16)) & 0x001f0000ff0000ffull;
-  x = (x | (x << 8)) & 0x100f00f00f00f00full;
-  x = (x | (x << 4)) & 0x10c30c30c30c30c3ull;
-  x = (x | (x << 2)) & 0x1249249249249249ull;
-  return x;
-}
-
-// Skilling's AxestoTranspose for 3 axes of b bits, written branch-free:
-// for each level Q (high to low), axis i either inverts the low bits of X0
-// (bit Q of Xi set) or exchanges the low bits of X0 and Xi; then Gray
-// encoding.  The index is the transposed bits read MSB first, i.e. bit q of
-// X0, X1, X2 at index bits 3q+2, 3q+1, 3q.
-__device__ __forceinline__ unsigned long long hilbert3(uint32_t x0, uint32_t x1, uint32_t x2, int b) {
-  for (int q = b - 1; q >= 1; --q) {
-    const uint32_t Q = 1u << q, P = Q - 1;
-    // axis 0: exchange with itself is a no-op, so only the inversion remains
-    x0 ^= P & (0u - ((x0 >> q) & 1u));
-    uint32_t m = 0u - ((x1 >> q) & 1u);
-    x0 ^= P & m;
-    uint32_t t = (x0 ^ x1) & P & ~m;
-    x0 ^= t; x1 ^= t;
-    m = 0u - ((x2 >> q) & 1u);
-    x0 ^= P & m;
-    t = (x0 ^ x2) & P & ~m;
-    x0 ^= t; x2 ^= t;
+// Skilling's AxestoTranspose + Gray encoding for 3 axes, read MSB first, as
+// a finite-state machine over the levels.  Level q's transformed bits y are
+// the raw bits r at level q mapped by the composition T of the exchange /
+// inversion steps of the levels above (each acts identically on every lower
+// bit position, so T is a map of 3-bit vectors); level q's own step is
+//   [y0: invert 0] [y1: invert 0 | else swap 0,1] [y2: invert 0 | else swap 0,2],
+// composed onto T for the levels below.  Gray: z = (y0, y1^y0, y2^y1^y0), and
+// the output digit is z ^ 111 when the parity p of z2 over the levels above
+// is odd (Skilling's t).  The states (T, p) reachable from (identity, 0) are
+// 48; the tables are built at compile time:
+//   t1[s][r]       = next state << 3 | digit                       (one level)
+//   t2[s][a0a1a2]  = state after two levels << 6 | digit_hi << 3 | digit_lo,
+// column a0 << 4 | a1 << 2 | a2 with a_i the two bits of axis i (high, low).
+// Checked against the oracle's Skilling transform bit for bit (GPU parity
+// tests, every b in [1, 21]).
+struct HilbertFsm {
+  uint16_t t2[48 * 64];
+  uint8_t t1[48 * 8];
+  int nstates;
+};
+struct HilbertState {
+  uint8_t v[8];  // T as a table of 3-bit vectors
+  uint8_t p;
+};
+constexpr uint8_t hilbert_level_op(uint8_t y, uint8_t v) {
+  int v0 = (v >> 2) & 1, v1 = (v >> 1) & 1, v2 = v & 1, t = 0;
+  if ((y >> 2) & 1) v0 ^= 1;
+  if ((y >> 1) & 1) {
+    v0 ^= 1;
+  } else {
+    t = v0; v0 = v1; v1 = t;
   }
-  x1 ^= x0;
-  x2 ^= x1;
-  uint32_t t = 0;
-  for (int q = b - 1; q >= 1; --q) t ^= ((x2 >> q) & 1u) ? ((1u << q) - 1u) : 0u;
-  x0 ^= t; x1 ^= t; x2 ^= t;
-  return (spread3(x0) << 2) | (spread3(x1) << 1) | spread3(x2);
+  if (y & 1) {
+    v0 ^= 1;
+  } else {
+    t = v0; v0 = v2; v2 = t;
+  }
+  return uint8_t((v0 << 2) | (v1 << 1) | v2);
+}
+constexpr HilbertFsm make_hilbert_fsm() {
+  HilbertFsm f{};
+  HilbertState st[64]{};
+  uint8_t nxt[64][8]{}, out[64][8]{};
+  for (int r = 0; r < 8; ++r) st[0].v[r] = uint8_t(r);
+  int ns = 1;
+  for (int i = 0; i < ns && ns <= 48; ++i) {
+    for (int r = 0; r < 8; ++r) {
+      const uint8_t y = st[i].v[r];
+      const int z0 = (y >> 2) & 1, z1 = ((y >> 1) & 1) ^ z0, z2 = (y & 1) ^ z1;
+      out[i][r] = uint8_t(((z0 << 2) | (z1 << 1) | z2) ^ (st[i].p ? 7 : 0));
+      HilbertState m{};
+      for (int k = 0; k < 8; ++k) m.v[k] = hilbert_level_op(y, st[i].v[k]);
+      m.p = uint8_t(st[i].p ^ z2);
+      int j = 0;
+      for (; j < ns; ++j) {
+        bool eq = st[j].p == m.p;
+        for (int k = 0; k < 8; ++k) eq = eq && st[j].v[k] == m.v[k];
+        if (eq) break;
+      }
+      if (j == ns && ns < 64) st[ns++] = m;
+      nxt[i][r] = uint8_t(j);
+    }
+  }
+  f.nstates = ns;
+  for (int i = 0; i < ns && i < 48; ++i) {
+    for (int r = 0; r < 8; ++r) f.t1[i * 8 + r] = uint8_t(nxt[i][r] << 3 | out[i][r]);
+    for (int c = 0; c < 64; ++c) {
+      const int a0 = (c >> 4) & 3, a1 = (c >> 2) & 3, a2 = c & 3;
+      const int rh = ((a0 >> 1) << 2) | ((a1 >> 1) << 1) | (a2 >> 1);
+      const int rl = ((a0 & 1) << 2) | ((a1 & 1) << 1) | (a2 & 1);
+      const int s1 = nxt[i][rh];
+      f.t2[i * 64 + c] = uint16_t(nxt[s1][rl] << 6 | out[i][rh] << 3 | out[s1][rl]);
+    }
+  }
+  return f;
+}
+constexpr HilbertFsm kHilbertFsm = make_hilbert_fsm();
+static_assert(kHilbertFsm.nstates == 48, "Skilling's 3-D transform has 48 (T, parity) states");
+__device__ const HilbertFsm g_hilbert_fsm = kHilbertFsm;
+
+// The key of cell (x0, x1, x2) at b bits per axis, tables in shared memory.
+template <class K>
+__host__ __device__ __forceinline__ K hilbert_key(uint32_t x0, uint32_t x1, uint32_t x2, int b, const uint16_t* t2,
+                                         const uint8_t* t1) {
+  uint32_t s = 0;
+  K key = 0;
+  int q = b;
+  if (q & 1) {  // odd b: the top level alone
+    --q;
+    const uint32_t e = t1[((x0 >> q) & 1u) << 2 | ((x1 >> q) & 1u) << 1 | ((x2 >> q) & 1u)];
+    key = K(e & 7u);
+    s = e >> 3;
+  }
+  while (q > 0) {
+    q -= 2;
+    const uint32_t c = ((x0 >> q) & 3u) << 4 | ((x1 >> q) & 3u) << 2 | ((x2 >> q) & 3u);
+    const uint32_t e = t2[s * 64 + c];
+    key = key << 6 | K(e & 63u);
+    s = e >> 6;
+  }
+  return key;
 }
 
 constexpr int kKeysThreads = 256;
@@ -210,7 +275,12 @@ __global__ __launch_bounds__(kKeysThreads) void k_keys(const V4* __restrict__ pm
                                                        uint32_t* __restrict__ ghist, int passes) {
   constexpr bool kF64 = sizeof(V4) == 32;  // NEXT-2: fp64 bodies, fp64 box
   __shared__ uint32_t sh[8 * 256];
+  __shared__ uint16_t ht2[48 * 64];
+  __shared__ uint8_t ht1[48 * 8];
   for (int i = threadIdx.x; i < passes * 256; i += kKeysThreads) sh[i] = 0;
+  for (int i = threadIdx.x; i < 48 * 64 / 2; i += kKeysThreads)
+    reinterpret_cast<uint32_t*>(ht2)[i] = reinterpret_cast<const uint32_t*>(g_hilbert_fsm.t2)[i];
+  for (int i = threadIdx.x; i < 48 * 8; i += kKeysThreads) ht1[i] = g_hilbert_fsm.t1[i];
   __syncthreads();
   const GridInfo g = *gi;
   const uint32_t qmax = (1u << g.b) - 1u;
@@ -229,7 +299,7 @@ __global__ __launch_bounds__(kKeysThreads) void k_keys(const V4* __restrict__ pm
       const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), l0), g.inv)));
       const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), l1), g.inv)));
       const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), l2), g.inv)));
-      key = K(hilbert3(q0, q1, q2, g.b));
+      key = hilbert_key<K>(q0, q1, q2, g.b, ht2, ht1);
       keys[i] = key;
     }
     const uint32_t act = __ballot_sync(0xffffffffu, ok);

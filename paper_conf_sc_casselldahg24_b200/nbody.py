@@ -126,6 +126,24 @@ class NBody:
         p, v, m = _f32(pos, self.n, 3), _f32(vel, self.n, 3), _f32(mass, self.n, 1)
         self._ck(self.lib.nbody_set_bodies(self.h, _ptr(p), _ptr(v), _ptr(m)))
 
+    def set_bodies_async(self, pos, vel, mass):
+        """nbody_set_bodies_async: the copy runs on the copy stream and overlaps
+        queued steps; `pos`, `vel`, `mass` (pinned host or device, fp32,
+        contiguous) must stay unchanged until sync()."""
+        if self.precision == 64:
+            raise ValueError("set_bodies_async is fp32 only")
+        self._keep_in = (_f32(pos, self.n, 3), _f32(vel, self.n, 3), _f32(mass, self.n, 1))
+        p, v, m = self._keep_in
+        self._ck(self.lib.nbody_set_bodies_async(self.h, _ptr(p), _ptr(v), _ptr(m)))
+
+    def get_positions_async(self, out):
+        """nbody_get_positions_async into out[n][3] (pinned host or device fp32,
+        contiguous); valid after sync()."""
+        o = _f32(out, self.n, 3)
+        if _ptr(o) != _ptr(out):
+            raise ValueError("get_positions_async needs a contiguous float32 [n, 3] output")
+        self._ck(self.lib.nbody_get_positions_async(self.h, _ptr(o)))
+
     def compute_accel(self):
         self._ck(self.lib.nbody_compute_accel(self.h))
 

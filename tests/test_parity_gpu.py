@@ -80,6 +80,19 @@ CASES = [
 ]
 
 
+@pytest.mark.parametrize("bits", list(range(1, 22)))
+def test_keys_every_grid_resolution(NB, oracle, bits):
+    """K2's table-driven Skilling automaton equals the oracle's transform at
+    every b (odd b takes the single-level table at the top), and K3's
+    permutation follows."""
+    pos, vel, mass = generate("clustered", 6001, 8)
+    sim = _run_gpu(NB, pos, vel, mass, 0.5, bits)
+    ref = oracle.step(pos, vel, mass, theta=0.5, eps=EPS, dt=DT, key_bits=bits, integrate=False,
+                      targets=np.array([0, 6000]))
+    assert (sim.debug_keys() == ref.keys).all()
+    assert (sim.debug_perm() == ref.perm).all()
+
+
 @pytest.mark.parametrize("name,n,seed,theta,bits", CASES)
 def test_force_pass_parity(NB, oracle, name, n, seed, theta, bits):
     pos, vel, mass = generate(name, n, seed)
