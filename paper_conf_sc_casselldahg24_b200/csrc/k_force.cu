@@ -417,6 +417,13 @@ constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 #ifndef NBODY_CAP_P
 #define NBODY_CAP_P 64
 #endif
+#ifndef NBODY_FUNROLL
+#define NBODY_FUNROLL 2
+#endif
+#ifndef NBODY_PUNROLL
+#define NBODY_PUNROLL 2
+#endif
+constexpr int kFUnroll = NBODY_FUNROLL, kPUnroll = NBODY_PUNROLL;  // dense loop unrolling (#pragma takes no macros)
 #ifndef NBODY_LEAF_DIRECT
 #define NBODY_LEAF_DIRECT 1
 #endif
@@ -560,7 +567,7 @@ __device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Targe
     }
     const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
     float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
-#pragma unroll 2
+#pragma unroll kFUnroll
     for (int p = 0; p < (nf + 1) >> 1; ++p) {
       const RecPair s = S.frec[p];
       interact2<kSoft>(ax, ay, az, s, s.m, nx, ny, nz, e2);
@@ -594,7 +601,7 @@ __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Targe
     const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
     float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
     uint32_t cnt = 0;
-#pragma unroll 2
+#pragma unroll kPUnroll
     for (int p = 0; p < (np + 1) >> 1; ++p) {
       const RecPair s = S.prec[p];
       const uint2 mk = *reinterpret_cast<const uint2*>(&S.pmsk[2 * p]);
