@@ -429,6 +429,11 @@ constexpr int kFUnroll = NBODY_FUNROLL, kPUnroll = NBODY_PUNROLL;  // dense loop
 #endif
 constexpr int kCapF = NBODY_CAP_F;  // dense list: entries every active lane interacts with
 constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
+// NEXT-4 quadrupole variant: the staged second moments (32 B per entry) make
+// the lists larger, so the full list and the T stack are shortened to keep 5
+// blocks per SM (measured: 70.3 ms at 4 blocks, 66.8 at 5, uniform 1e7).
+template <bool kQuad> constexpr int cap_f() { return kQuad ? 64 : kCapF; }
+template <bool kQuad> constexpr int cap_t() { return kQuad ? 224 : kCapT; }
 
 // Records in pairs, component-interleaved, so that one 16-B shared load
 // yields (x_a, x_b, y_a, y_b) and the interaction of two entries runs on the
@@ -442,9 +447,19 @@ struct alignas(16) RecPair {
     reinterpret_cast<float*>(&z)[h] = r.z;
     reinterpret_cast<float*>(&m)[h] = r.w;
   }
-  __device__ __forceinline__ float4 get(int h) const {
-    return make_float4(reinterpret_cast<const float*>(&x)[h], reinterpret_cast<const float*>(&y)[h],
-                       reinterpret_cast<const float*>(&z)[h], reinterpret_cast<const float*>(&m)[h]);
+};
+// NEXT-4 [A24]: the fp32 second moments of two entries, component-
+// interleaved like RecPair (qf layout: (Sxx, Syy, Szz, trS), (Sxy, Sxz, Syz)).
+struct alignas(16) QuadPair {
+  float2 xx, yy, zz, tr, xy, xz, yz, pad;
+  __device__ __forceinline__ void put(int h, const float4& q0, const float4& q1) {
+    reinterpret_cast<float*>(&xx)[h] = q0.x;
+    reinterpret_cast<float*>(&yy)[h] = q0.y;
+    reinterpret_cast<float*>(&zz)[h] = q0.z;
+    reinterpret_cast<float*>(&tr)[h] = -1.5f * q0.w;  // -(3/2) tr S, pre-scaled for the radial coefficient
+    reinterpret_cast<float*>(&xy)[h] = q1.x;
+    reinterpret_cast<float*>(&xz)[h] = q1.y;
+    reinterpret_cast<float*>(&yz)[h] = q1.z;
   }
 };
 // Targets in pairs for the transposed test, relative to the group reference
@@ -459,15 +474,17 @@ struct alignas(16) V0Smem {
   TgtPair tgt[16];          // the warp's targets for the transposed test (paired)
   float4 tpos[kF64 ? 1 : 32];   // the warp's target positions (fp64 fallback)
   double4 tpos64[kF64 ? 32 : 1];  // NEXT-2 FP64 mode: exact target positions
-  RecPair frec[kF64 ? 1 : kCapF / 2];  // monopole / body records, all lanes
+  static constexpr int kF = cap_f<kQuad>(), kT = cap_t<kQuad>();
+  RecPair frec[kF64 ? 1 : kF / 2];  // monopole / body records, all lanes
   RecPair prec[kF64 ? 1 : kCapP / 2];  // monopole / body records, ...
-  double4 frec64[kF64 ? kCapF : 1];    // NEXT-2 FP64 mode: the same lists in fp64
+  double4 frec64[kF64 ? kF : 1];    // NEXT-2 FP64 mode: the same lists in fp64
   double4 prec64[kF64 ? kCapP : 1];
   uint32_t pmsk[kCapP];     // ... for the lanes in the mask
   uint32_t astk[kCapA];
-  uint2 tstk[kCapT];     // (id, mask of the targets that reached it)
-  uint32_t fid[kQuad ? kCapF : 1];  // NEXT-4: node id of each entry (0: a body)
-  uint32_t pid[kQuad ? kCapP : 1];
+  uint2 tstk[kT];     // (id, mask of the targets that reached it)
+  using QP = typename std::conditional<kQuad, QuadPair, char>::type;
+  QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
+  QP pq[kQuad ? kCapP / 2 : 1];
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -549,17 +566,61 @@ __device__ __forceinline__ void interact2(float2& ax, float2& ay, float2& az, co
   az = __ffma2_rn(w, dz, az);
 }
 
+// Two monopole + quadrupole interactions on the packed pipe [A24]: with
+// d = s - x and inv = (|d|^2 + eps^2)^(-1/2),
+//   a += {m inv^3 + [(15/2) d.S.d inv^2 - (3/2) tr(S)] inv^5} d - 3 (S d) inv^5.
+// `on` (per half) masks the whole term; bodies carry S = 0.
+template <bool kSoft>
+__device__ __forceinline__ void interact2_quad(float2& ax, float2& ay, float2& az, const RecPair& s,
+                                               const QuadPair& q, bool on0, bool on1, float2 nx, float2 ny,
+                                               float2 nz, float2 eps2) {
+  const float2 dx = __fadd2_rn(s.x, nx), dy = __fadd2_rn(s.y, ny), dz = __fadd2_rn(s.z, nz);
+  const float2 r2 = __ffma2_rn(dz, dz, __ffma2_rn(dy, dy, __ffma2_rn(dx, dx, eps2)));
+  float2 inv = make_float2(rsqrt_fast(r2.x), rsqrt_fast(r2.y));
+  if (!kSoft) {
+    inv.x = r2.x > 0.f ? inv.x : 0.f;
+    inv.y = r2.y > 0.f ? inv.y : 0.f;
+  }
+  const float2 inv2 = __fmul2_rn(inv, inv);
+  const float2 inv3 = __fmul2_rn(inv2, inv);
+  const float2 inv5 = __fmul2_rn(inv3, inv2);
+  const float2 sx = __ffma2_rn(q.xx, dx, __ffma2_rn(q.xy, dy, __fmul2_rn(q.xz, dz)));
+  const float2 sy = __ffma2_rn(q.xy, dx, __ffma2_rn(q.yy, dy, __fmul2_rn(q.yz, dz)));
+  const float2 sz = __ffma2_rn(q.xz, dx, __ffma2_rn(q.yz, dy, __fmul2_rn(q.zz, dz)));
+  const float2 dsd = __ffma2_rn(dx, sx, __ffma2_rn(dy, sy, __fmul2_rn(dz, sz)));
+  // radial coefficient m inv^3 + [(15/2) dsd inv^2 - (3/2) tr] inv^5 (q.tr holds -(3/2) tr S)
+  const float2 t = __ffma2_rn(dsd, __fmul2_rn(f2(7.5f), inv2), q.tr);
+  float2 cw = __ffma2_rn(t, inv5, __fmul2_rn(s.m, inv3));
+  float2 e = __fmul2_rn(f2(-3.f), inv5);
+  cw = make_float2(on0 ? cw.x : 0.f, on1 ? cw.y : 0.f);
+  e = make_float2(on0 ? e.x : 0.f, on1 ? e.y : 0.f);
+  ax = __ffma2_rn(cw, dx, __ffma2_rn(e, sx, ax));
+  ay = __ffma2_rn(cw, dy, __ffma2_rn(e, sy, ay));
+  az = __ffma2_rn(cw, dz, __ffma2_rn(e, sz, az));
+}
+
 // Entries [0, cnt) of a pair list; an odd count is padded with a massless
 // entry (it adds exactly 0).
 template <bool kSoft, bool kQuad>
 __device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Target& T, Acc& a, const float4* qf,
                                            int lane) {
-  if (kQuad) {
-#pragma unroll 4
-    for (int e = 0; e < nf; ++e) {
-      const float4 s = S.frec[e >> 1].get(e & 1);
-      interact<kSoft, kQuad>(a, s, s.w, T, qf, S.fid[e], true);
+  if constexpr (kQuad) {
+    if (nf & 1) {
+      if (lane == 0) {
+        S.frec[nf >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f));
+        S.fq[nf >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f), make_float4(0.f, 0.f, 0.f, 0.f));
+      }
+      __syncwarp();
     }
+    const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
+    float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
+    for (int p = 0; p < (nf + 1) >> 1; ++p) {
+      const RecPair s = S.frec[p];
+      interact2_quad<kSoft>(ax, ay, az, s, S.fq[p], true, true, nx, ny, nz, e2);
+    }
+    a.x += ax.x + ax.y;
+    a.y += ay.x + ay.y;
+    a.z += az.x + az.y;
   } else {
     if (nf & 1) {
       if (lane == 0) S.frec[nf >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f));
@@ -582,14 +643,29 @@ __device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Targe
 template <bool kSoft, bool kQuad>
 __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane,
                                            const float4* qf) {
-  if (kQuad) {
-#pragma unroll 4
-    for (int e = 0; e < np; ++e) {
-      const float4 s = S.prec[e >> 1].get(e & 1);
-      const bool on = (S.pmsk[e] >> lane) & 1u;
-      interact<kSoft, kQuad>(a, s, on ? s.w : 0.f, T, qf, S.pid[e], on);
-      a.n += on;
+  if constexpr (kQuad) {
+    if (np & 1) {
+      if (lane == 0) {
+        S.prec[np >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f));
+        S.pq[np >> 1].put(1, make_float4(0.f, 0.f, 0.f, 0.f), make_float4(0.f, 0.f, 0.f, 0.f));
+        S.pmsk[np] = 0u;
+      }
+      __syncwarp();
     }
+    const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
+    float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
+    uint32_t cnt = 0;
+    for (int p = 0; p < (np + 1) >> 1; ++p) {
+      const RecPair s = S.prec[p];
+      const uint2 mk = *reinterpret_cast<const uint2*>(&S.pmsk[2 * p]);
+      const bool on0 = (mk.x >> lane) & 1u, on1 = (mk.y >> lane) & 1u;
+      interact2_quad<kSoft>(ax, ay, az, s, S.pq[p], on0, on1, nx, ny, nz, e2);
+      cnt += uint32_t(on0) + uint32_t(on1);
+    }
+    a.x += ax.x + ax.y;
+    a.y += ay.x + ay.y;
+    a.z += az.x + az.y;
+    a.n += cnt;
   } else {
     if (np & 1) {
       if (lane == 0) {
@@ -723,13 +799,20 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     const bool part = want && msk != amask;
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
+    float4 q0 = make_float4(0.f, 0.f, 0.f, 0.f), q1 = q0;  // NEXT-4: the node's moments (0 for a body)
+    if constexpr (kQuad) {
+      if ((full || part) && id) {
+        q0 = __ldg(qf + 2 * size_t(id));
+        q1 = __ldg(qf + 2 * size_t(id) + 1);
+      }
+    }
     if (full) {
       const int pos = nf + __popc(bf & lt);
       if constexpr (kF64)
         S.frec64[pos] = P.t.rec64[g];
       else
         S.frec[pos >> 1].put(pos & 1, r);
-      if (kQuad) S.fid[pos] = id;
+      if constexpr (kQuad) S.fq[pos >> 1].put(pos & 1, q0, q1);
     }
     if (part) {
       const int pos = np + __popc(bp & lt);
@@ -738,7 +821,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       else
         S.prec[pos >> 1].put(pos & 1, r);
       S.pmsk[pos] = msk;
-      if (kQuad) S.pid[pos] = id;
+      if constexpr (kQuad) S.pq[pos >> 1].put(pos & 1, q0, q1);
     }
     nf += __popc(bf);
     np += __popc(bp);
@@ -772,7 +855,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   };
   auto flush = [&](bool all) {
     __syncwarp();
-    if (nf > kCapF - 32 || (all && nf > 0)) {
+    if (nf > S.kF - 32 || (all && nf > 0)) {
       if constexpr (kF64)
         dense_full64<kSoft>(S, nf, T, a);
       else
@@ -901,10 +984,10 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
         flush(false);
         append(mb != 0u, rb, mb, 0u, cb);
       }
-      const bool push = rm != 0u && nt + 64 <= kCapT && !lv;
-      const bool room = nt + 64 <= kCapT || lv;
+      const bool push = rm != 0u && nt + 64 <= S.kT && !lv;
+      const bool room = nt + 64 <= S.kT || lv;
 #else
-      const bool room = nt + 64 <= kCapT;
+      const bool room = nt + 64 <= S.kT;
       const bool push = rm != 0u && room;
 #endif
       const uint32_t b1 = __ballot_sync(kFull, push);
