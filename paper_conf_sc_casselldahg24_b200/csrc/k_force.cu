@@ -432,8 +432,11 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 // NEXT-4 quadrupole variant: the staged second moments (32 B per entry) make
 // the lists larger, so the full list and the T stack are shortened to keep 5
 // blocks per SM (measured: 70.3 ms at 4 blocks, 66.8 at 5, uniform 1e7).
-template <bool kQuad> constexpr int cap_f() { return kQuad ? 64 : kCapF; }
-template <bool kQuad> constexpr int cap_t() { return kQuad ? 224 : kCapT; }
+// NEXT-2 FP64 mode (32-B fp64 records): 64 full entries, 192 T slots and at
+// most 72 registers give 6 blocks per SM (disks 1e7: 67.7 ms at 4 blocks with
+// 124 registers, 58.0 ms here; 128 T slots overflow too often: 75.9 ms).
+template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad || kF64 ? 64 : kCapF; }
+template <bool kQuad, bool kF64> constexpr int cap_t() { return kQuad ? 224 : kF64 ? 192 : kCapT; }
 
 // Records in pairs, component-interleaved, so that one 16-B shared load
 // yields (x_a, x_b, y_a, y_b) and the interaction of two entries runs on the
@@ -474,7 +477,7 @@ struct alignas(16) V0Smem {
   TgtPair tgt[16];          // the warp's targets for the transposed test (paired)
   float4 tpos[kF64 ? 1 : 32];   // the warp's target positions (fp64 fallback)
   double4 tpos64[kF64 ? 32 : 1];  // NEXT-2 FP64 mode: exact target positions
-  static constexpr int kF = cap_f<kQuad>(), kT = cap_t<kQuad>();
+  static constexpr int kF = cap_f<kQuad, kF64_>(), kT = cap_t<kQuad, kF64_>();
   RecPair frec[kF64 ? 1 : kF / 2];  // monopole / body records, all lanes
   RecPair prec[kF64 ? 1 : kCapP / 2];  // monopole / body records, ...
   double4 frec64[kF64 ? kF : 1];    // NEXT-2 FP64 mode: the same lists in fp64
@@ -693,9 +696,14 @@ __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Targe
 }
 
 // NEXT-2 FP64 mode dense phase: fp64 records, fp64 arithmetic.
+#ifndef NBODY_F64_UNROLL
+#define NBODY_F64_UNROLL 2
+#endif
+constexpr int kUnroll64 = NBODY_F64_UNROLL;
+
 template <bool kSoft>
 __device__ __forceinline__ void dense_full64(V0Smem<false, true>& S, int nf, const Target& T, AccD& a) {
-#pragma unroll 2
+#pragma unroll kUnroll64
   for (int e = 0; e < nf; ++e) {
     const double4 s = S.frec64[e];
     interact64<kSoft>(a, s, s.w, T);
@@ -706,7 +714,7 @@ __device__ __forceinline__ void dense_full64(V0Smem<false, true>& S, int nf, con
 template <bool kSoft>
 __device__ __forceinline__ void dense_part64(V0Smem<false, true>& S, int np, const Target& T, AccD& a, int lane) {
   uint32_t cnt = 0;
-#pragma unroll 2
+#pragma unroll kUnroll64
   for (int e = 0; e < np; ++e) {
     const double4 s = S.prec64[e];
     const bool on = (S.pmsk[e] >> lane) & 1u;
@@ -717,7 +725,7 @@ __device__ __forceinline__ void dense_part64(V0Smem<false, true>& S, int np, con
 }
 
 #ifndef NBODY_V0_MINB_F64
-#define NBODY_V0_MINB_F64 4
+#define NBODY_V0_MINB_F64 7
 #endif
 
 template <bool kSoft, bool kQuad, bool kF64>

@@ -20,10 +20,11 @@ ap.add_argument("--passes", type=int, default=2)
 ap.add_argument("--traversal", type=int, default=0)
 ap.add_argument("--key-bits", type=int, default=16)
 ap.add_argument("--multipole", type=int, default=1)
+ap.add_argument("--precision", type=int, default=32)
 a = ap.parse_args()
 pos, vel, mass = generate(a.workload, a.n, a.seed)
 sim = NBody(a.n, a.theta, 1e-3, 1e-3, key_bits=a.key_bits, use_graph=False, traversal=a.traversal,
-            multipole=a.multipole)
+            multipole=a.multipole, precision=a.precision)
 sim.set_option(5, 1)
 sim.set_bodies(pos, vel, mass)
 for _ in range(a.passes):
