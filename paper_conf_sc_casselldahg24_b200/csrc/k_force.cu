@@ -435,8 +435,14 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 // NEXT-2 FP64 mode (32-B fp64 records): 64 full entries, 192 T slots and at
 // most 72 registers give 6 blocks per SM (disks 1e7: 67.7 ms at 4 blocks with
 // 124 registers, 58.0 ms here; 128 T slots overflow too often: 75.9 ms).
-template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad || kF64 ? 64 : kCapF; }
-template <bool kQuad, bool kF64> constexpr int cap_t() { return kQuad ? 224 : kF64 ? 192 : kCapT; }
+#ifndef NBODY_QCAP_F
+#define NBODY_QCAP_F 64
+#endif
+#ifndef NBODY_QCAP_T
+#define NBODY_QCAP_T 224
+#endif
+template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad ? NBODY_QCAP_F : kF64 ? 64 : kCapF; }
+template <bool kQuad, bool kF64> constexpr int cap_t() { return kQuad ? NBODY_QCAP_T : kF64 ? 192 : kCapT; }
 
 // Records in pairs, component-interleaved, so that one 16-B shared load
 // yields (x_a, x_b, y_a, y_b) and the interaction of two entries runs on the
