@@ -92,8 +92,8 @@ __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, dou
   // d2 > (1 + 2e-4) s^2/theta^2 + A surely accepts and
   // d2 < (1 - 2e-4) s^2/theta^2 - A surely opens.
   float2 rc;
+  const double q = t.th2 > 0.0 ? __ddiv_rn(s2, t.th2) : 0.0;  // s^2 / theta^2, once per node
   if (t.th2 > 0.0) {
-    const double q = s2 / t.th2;
     const double A = double(t.grid->abs_d2);
     rc.x = __double2float_rd((1.0 - 2e-4) * q - A);
     rc.y = __double2float_ru((1.0 + 2e-4) * q + A);
@@ -108,7 +108,7 @@ __device__ __forceinline__ void finish_node(const TreeView& t, int64_t node, dou
   t.tf[node] = make_float4(__double2float_rn(__dsub_rn(c[0], double(c0))),
                            __double2float_rn(__dsub_rn(c[1], double(c1))),
                            __double2float_rn(__dsub_rn(c[2], double(c2))),
-                           t.th2 > 0.0 ? __double2float_rn(__ddiv_rn(s2, t.th2)) : __int_as_float(0x7f800000));
+                           t.th2 > 0.0 ? __double2float_rn(q) : __int_as_float(0x7f800000));
   if (S) {
     if (keep) {
 #pragma unroll
