@@ -217,9 +217,18 @@ def run_ours(args, cfg, world, rank, local):
 
     from paper_conf_sc_casselldahg24_b200 import NBody
 
+    # NBODY_BENCH_ONE_DEVICE=1 (validation of the N > 1 path on a one-GPU
+    # box only, never a reported number): every rank on GPU 0, gloo for the
+    # host-side plumbing; the exchange itself still runs over CUDA IPC.
+    one_device = world > 1 and os.environ.get("NBODY_BENCH_ONE_DEVICE") == "1"
+    if one_device:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_device:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     n = cfg["n"]
     f64 = args.precision == 64
     pos, vel, mass = generate(cfg["workload"], n, cfg["seed"], np.float64 if f64 else np.float32)
