@@ -71,3 +71,42 @@ def test_async_device_buffers_and_deferred_validation(NB):
     sim.set_bodies(pos, vel, mass)
     sim.step(1)
     sim.sync()
+
+
+@pytest.mark.parametrize("n", [1, 2, 33, 1025])
+def test_async_small_and_ragged(NB, n):
+    import torch
+    pos, vel, mass = generate("uniform", n, 11)
+    ref = NB(n, 0.5, 1e-3, 1e-3, key_bits=16)
+    ref.set_bodies(pos, vel, mass)
+    ref.compute_accel()
+    a_ref = ref.get_accel()
+    ref.set_bodies(pos, vel, mass)
+    ref.step(3)
+    x_ref = ref.get_positions()
+    sim = NB(n, 0.5, 1e-3, 1e-3, key_bits=16)
+    hp, hv, hm = (torch.from_numpy(a).pin_memory() for a in (pos, vel, mass))
+    sim.set_bodies_async(hp, hv, hm)
+    sim.compute_accel()
+    assert (sim.get_accel() == a_ref).all()  # a synchronous getter after an async load
+    sim.set_bodies_async(hp, hv, hm)
+    sim.step(3)
+    out = torch.empty((n, 3), dtype=torch.float32).pin_memory()
+    sim.get_positions_async(out)
+    sim.sync()
+    assert (out.numpy() == x_ref).all()
+
+
+def test_async_api_checks(NB):
+    import torch
+    n = 64
+    pos, vel, mass = generate("uniform", n, 12)
+    sim = NB(n, 0.5, 1e-3, 1e-3)
+    out = torch.empty((n, 3), dtype=torch.float32).pin_memory()
+    with pytest.raises(Exception):
+        sim.get_positions_async(out)  # nothing loaded yet
+    f64 = NB(n, 0.5, 1e-3, 1e-3, precision=64)
+    with pytest.raises(ValueError):
+        f64.set_bodies_async(pos, vel, mass)
+    st = f64.lib.nbody_set_bodies_async(f64.h, None, None, None)
+    assert st == -1  # NBODY_EINVAL
