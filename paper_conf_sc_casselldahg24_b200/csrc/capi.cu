@@ -387,7 +387,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
       launch_keys32(c->pm[0], n, c->grid, static_cast<uint32_t*>(c->keys[0]), c->sort.ghist, c->sort.passes, s);
     else
       launch_keys64(c->pm[0], n, c->grid, static_cast<unsigned long long*>(c->keys[0]), c->sort.ghist,
-                    c->sort.passes, s);
+                    c->sort.passes, c->b, s);
     if (debug) {
       CK(cudaMemcpyAsync(c->keys_dbg, c->keys[0], size_t(c->key_bytes) * n, cudaMemcpyDeviceToDevice, s));
     }

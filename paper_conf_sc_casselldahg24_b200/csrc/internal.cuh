@@ -105,7 +105,7 @@ void launch_bbox_final(const float* partial, int nparts, int b, GridInfo* g, cud
 void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* keys, uint32_t* ghist, int passes,
                    cudaStream_t s);
 void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
-                   int passes, cudaStream_t s);
+                   int passes, int b, cudaStream_t s);
 // NEXT-2 FP64 mode: the same stages on fp64 bodies (x, y, z, m) as double4;
 // partial[block][6] doubles; the grid's lo64/hi64 hold the box.
 void launch_bbox_partial_f64(const double4* pm, int64_t n, double* partial, int nblocks, cudaStream_t s);

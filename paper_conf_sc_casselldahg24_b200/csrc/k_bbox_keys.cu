@@ -240,18 +240,19 @@ static_assert(kHilbertFsm.nstates == 48, "Skilling's 3-D transform has 48 (T, pa
 __device__ const HilbertFsm g_hilbert_fsm = kHilbertFsm;
 
 // The key of cell (x0, x1, x2) at b bits per axis, tables in shared memory.
-template <class K>
+template <class K, int kB = 0>  // kB > 0: b fixed at compile time (unrolled, constant shifts)
 __host__ __device__ __forceinline__ K hilbert_key(uint32_t x0, uint32_t x1, uint32_t x2, int b, const uint16_t* t2,
                                          const uint8_t* t1) {
   uint32_t s = 0;
   K key = 0;
-  int q = b;
+  int q = kB > 0 ? kB : b;
   if (q & 1) {  // odd b: the top level alone
     --q;
     const uint32_t e = t1[((x0 >> q) & 1u) << 2 | ((x1 >> q) & 1u) << 1 | ((x2 >> q) & 1u)];
     key = K(e & 7u);
     s = e >> 3;
   }
+#pragma unroll
   while (q > 0) {
     q -= 2;
     const uint32_t c = ((x0 >> q) & 3u) << 4 | ((x1 >> q) & 3u) << 2 | ((x2 >> q) & 3u);
@@ -269,10 +270,13 @@ constexpr int kKeysThreads = 256;
 // sort passes).  Grid-stride; per-block shared histograms; a warp whose 32
 // keys share a digit adds it once (common for the high digits: the input is
 // the previous step's Hilbert order).
-template <class K, class V4>
+// kB, kPasses > 0: the grid resolution and radix passes fixed at compile time
+// (the default b = 16: 48-bit keys, 6 passes); 0: read at run time.
+template <class K, class V4, int kB = 0, int kPasses = 0>
 __global__ __launch_bounds__(kKeysThreads) void k_keys(const V4* __restrict__ pm, int64_t n,
                                                        const GridInfo* __restrict__ gi, K* __restrict__ keys,
-                                                       uint32_t* __restrict__ ghist, int passes) {
+                                                       uint32_t* __restrict__ ghist, int passes_rt) {
+  const int passes = kPasses > 0 ? kPasses : passes_rt;
   constexpr bool kF64 = sizeof(V4) == 32;  // NEXT-2: fp64 bodies, fp64 box
   __shared__ uint32_t sh[8 * 256];
   __shared__ uint16_t ht2[48 * 64];
@@ -299,11 +303,12 @@ __global__ __launch_bounds__(kKeysThreads) void k_keys(const V4* __restrict__ pm
       const uint32_t q0 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.x), l0), g.inv)));
       const uint32_t q1 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.y), l1), g.inv)));
       const uint32_t q2 = min(qmax, __double2uint_rz(__dmul_rn(__dsub_rn(double(p.z), l2), g.inv)));
-      key = hilbert_key<K>(q0, q1, q2, g.b, ht2, ht1);
+      key = hilbert_key<K, kB>(q0, q1, q2, g.b, ht2, ht1);
       keys[i] = key;
     }
     const uint32_t act = __ballot_sync(0xffffffffu, ok);
-    for (int ps = 0; ps < passes; ++ps) {
+#pragma unroll
+    for (int ps = 0; ps < (kPasses > 0 ? kPasses : passes); ++ps) {
       const uint32_t d = uint32_t(key >> (8 * ps)) & 255u;
       const uint32_t d0 = __shfl_sync(0xffffffffu, d, 0);
       if (__all_sync(0xffffffffu, !ok || d == d0)) {
@@ -340,8 +345,11 @@ void launch_keys32(const float4* pm, int64_t n, const GridInfo* g, uint32_t* key
 }
 
 void launch_keys64(const float4* pm, int64_t n, const GridInfo* g, unsigned long long* keys, uint32_t* ghist,
-                   int passes, cudaStream_t s) {
-  k_keys<unsigned long long><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
+                   int passes, int b, cudaStream_t s) {
+  if (b == 16 && passes == 6)  // the default grid
+    k_keys<unsigned long long, float4, 16, 6><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
+  else
+    k_keys<unsigned long long><<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, keys, ghist, passes);
 }
 
 void launch_bbox_partial_f64(const double4* pm, int64_t n, double* partial, int nblocks, cudaStream_t s) {
