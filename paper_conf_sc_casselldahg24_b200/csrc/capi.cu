@@ -789,14 +789,11 @@ nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, 
 static nbody_status ensure_xfer(nbody_ctx* c) {
   if (c->xfer) return NBODY_OK;
   const size_t n = size_t(c->n);
-  CK(cudaStreamCreateWithFlags(&c->cstream, cudaStreamNonBlocking));
-  CK(cudaStreamCreateWithFlags(&c->ostream, cudaStreamNonBlocking));
-  for (int k = 0; k < 2; ++k) {
-    CK(cudaEventCreateWithFlags(&c->ev_in_copied[k], cudaEventDisableTiming));
-    CK(cudaEventCreateWithFlags(&c->ev_in_used[k], cudaEventDisableTiming));
-    CK(cudaEventCreateWithFlags(&c->ev_out_ready[k], cudaEventDisableTiming));
-    CK(cudaEventCreateWithFlags(&c->ev_out_copied[k], cudaEventDisableTiming));
-  }
+  if (!c->cstream) CK(cudaStreamCreateWithFlags(&c->cstream, cudaStreamNonBlocking));
+  if (!c->ostream) CK(cudaStreamCreateWithFlags(&c->ostream, cudaStreamNonBlocking));
+  for (int k = 0; k < 2; ++k)
+    for (cudaEvent_t* e : {&c->ev_in_copied[k], &c->ev_in_used[k], &c->ev_out_ready[k], &c->ev_out_copied[k]})
+      if (!*e) CK(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
   void* p = nullptr;
   const cudaError_t e = cudaMalloc(&p, align_up(2 * 28 * n) + align_up(2 * 12 * n) + 256);
   if (e != cudaSuccess) {

@@ -17,6 +17,8 @@
 //     of a tile are runs of consecutive addresses.
 // HBM bound: per pass 2 x (key + 4 B) per body; the upfront histogram reads
 // the keys once.
+#include <atomic>
+
 #include <cuda/atomic>
 
 #include "internal.cuh"
@@ -255,11 +257,15 @@ void set_attr() {
 
 template <class K>
 void run_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s) {
-  static bool attrs = false;
-  if (!attrs) {
+  // the dynamic shared-memory opt-in is a per-device function attribute
+  static std::atomic<uint64_t> attrs_done{0};  // bit d: set on device d
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = uint64_t(1) << (dev & 63);
+  if (!(attrs_done.load() & bit)) {
     set_attr<K, true, true>(); set_attr<K, true, false>();
     set_attr<K, false, true>(); set_attr<K, false, false>();
-    attrs = true;
+    attrs_done.fetch_or(bit);
   }
   cudaMemsetAsync(p.tile_ctr, 0, sizeof(uint32_t) * 8, s);
   cudaMemsetAsync(p.status, 0, sizeof(uint32_t) * size_t(p.passes) * size_t(p.tiles) * kRadix, s);
