@@ -534,7 +534,8 @@ nbody_status sync_stream(nbody_ctx* c) {
   CK(cudaStreamSynchronize(c->stream));
   if (c->xpeer) {
     int err = 0;
-    CK(cudaMemcpy(&err, c->xerr, sizeof(int), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpyAsync(&err, c->xerr, sizeof(int), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
     if (err) {
       c->state = NBODY_ESTATE;
       c->err = "peer exchange: a barrier timed out (a rank stopped stepping); the state is invalid";
@@ -903,9 +904,10 @@ nbody_status nbody_sync(nbody_ctx* c) {
   const nbody_status st = sync_stream(c);
   if (st != NBODY_OK || !c->bad_async) return st;
   int bad = 0;
-  CK(cudaMemcpy(&bad, c->bad_async, sizeof(int), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpyAsync(&bad, c->bad_async, sizeof(int), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
   if (bad) {
-    CK(cudaMemset(c->bad_async, 0, sizeof(int)));
+    CK(cudaMemsetAsync(c->bad_async, 0, sizeof(int), c->stream));
     c->loaded = false;
     return fail(c, NBODY_EINVAL, (bad & 2) ? "an async input set had masses that are not finite and > 0"
                                            : "an async input set had a non-finite position or velocity");
