@@ -66,7 +66,10 @@ enum {
    * launches. */
   NBODY_OPT_USE_GRAPH = 3,
   /* CALCULATEFORCE kernel variant: 0 = default (fastest validated),
-   * 1 = warp mask-stack walk (per-lane exact lists, no group lists). */
+   * 1 = warp mask-stack walk (per-lane exact lists, no group lists),
+   * 2 = the paper's scheme: one thread per body, stackless skip-list DFS
+   * (monopole only).  All three give the same interaction
+   * lists. */
   NBODY_OPT_TRAVERSAL = 4,
   /* 1 = record CUDA events around each stage of a pass issued by
    * nbody_compute_accel / nbody_step with graphs off; nbody_get_stats then

@@ -656,6 +656,7 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
     case NBODY_OPT_MULTIPOLE:
       if (value != 1 && value != 2) return fail(c, NBODY_EINVAL, "multipole order must be 1 or 2");
       if (value == 2 && c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode is monopole only");
+      if (value == 2 && c->traversal == 2) return fail(c, NBODY_EINVAL, "traversal variant 2 is monopole only");
       if (value == 2 && !c->tree.S64) {  // allocated on first use: 80 B per internal id
         const size_t inner = size_t(1) << c->tree.L;
         cudaError_t e = cudaMalloc(&c->quad_arena, 48 * inner + 32 * inner);
@@ -702,8 +703,9 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       drop_graph(c);
       return NBODY_OK;
     case NBODY_OPT_TRAVERSAL:
-      if (value < 0 || value > 1) return fail(c, NBODY_EINVAL, "unknown traversal variant");
+      if (value < 0 || value > 2) return fail(c, NBODY_EINVAL, "unknown traversal variant");
       if (value != 0 && c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode uses traversal variant 0");
+      if (value == 2 && c->tree.quad) return fail(c, NBODY_EINVAL, "traversal variant 2 is monopole only");
       c->traversal = int(value);
       drop_graph(c);
       return NBODY_OK;

@@ -398,6 +398,59 @@ __global__ __launch_bounds__(32 * kV1Warps) void k_force_maskstack(const ForcePa
 }
 
 
+// ------------------------------------------------------------ variant 2 ----
+// The paper's own CALCULATEFORCE scheme, for comparison: one thread per
+// target body walking the BVH depth-first without a stack by the skip-list
+// jumps of P:222 / P:245 [A7] -- cursor (l, s) = the node of level l whose
+// first leaf is s; open: l <- l - 1; done with a node: s <- s + 2^l, stop at
+// s >= N, else l <- min(ctz(s), L).  The decisions are the same fp32-filtered
+// fp64 test per lane (no warp votes: lanes diverge freely), so the lists --
+// and the counts -- equal the other variants'.  Monopole only.
+constexpr int kV2Threads = 256;
+
+__global__ __launch_bounds__(kV2Threads) void k_force_skiplist(const ForceParams P) {
+  const int lane = threadIdx.x & 31;
+  int64_t tb, te;
+  owned_range(P, tb, te);
+  const int64_t k0 = tb + int64_t(blockIdx.x) * kV2Threads + (threadIdx.x & ~31);
+  const int64_t k = k0 + lane;
+  const bool active = k < te;
+  const Target T = load_target(P, k, active);
+  const Walk W = make_walk(P);
+  const uint32_t kid = W.leaf0 + uint32_t(k);
+  Acc a;
+  int l = W.L;
+  uint32_t sl = 0;  // first leaf of the current node
+  while (active) {
+    const uint32_t g = (W.leaf0 + sl) >> l;
+    const float4 r = __ldg(W.rec + g);
+    const Probe pr = probe(r, T);
+    bool take;  // interact with this node and skip its subtree
+    if (l == 0) {
+      take = true;
+      const bool on = g != kid;  // a leaf never acts on itself
+      a.add(on, pr.dx, pr.dy, pr.dz, pr.d2, r.w, T.eps2);
+      a.n += on;
+    } else {
+      const float2 c = __ldg(W.rc + g);
+      take = pr.d2 > c.y;
+      if (!take && !(pr.d2 < c.x)) take = opening_accept64(W.pred[g], T.x, T.y, T.z, T.th2);
+      if (take) {
+        a.add(true, pr.dx, pr.dy, pr.dz, pr.d2, r.w, T.eps2);
+        ++a.n;
+      }
+    }
+    if (take) {
+      sl += 1u << l;
+      if (sl >= W.n) break;
+      l = min(__ffs(int(sl)) - 1, W.L);
+    } else {
+      --l;
+    }
+  }
+  store_result(P, tb, k, k0, active, a, lane);
+}
+
 // ------------------------------------------------------------ variant 0 ----
 constexpr int kV0Warps = 4;
 // Sized for 8 blocks x 4 warps per SM (26.4 KB shared memory per block);
@@ -1106,7 +1159,9 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
   if (nt <= 0) return;
   const int64_t warps = (nt + 31) / 32;
   const bool quad = p.t.quad;
-  if (variant == 1) {
+  if (variant == 2) {  // the paper's per-body skip-list walk (monopole)
+    k_force_skiplist<<<unsigned((nt + kV2Threads - 1) / kV2Threads), kV2Threads, 0, s>>>(p);
+  } else if (variant == 1) {
     const unsigned grid = unsigned((warps + kV1Warps - 1) / kV1Warps);
     if (quad)
       k_force_maskstack<true><<<grid, 32 * kV1Warps, 0, s>>>(p);

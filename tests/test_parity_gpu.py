@@ -135,6 +135,32 @@ def test_traversal_variants_agree(NB, oracle):
     assert e.max() < 1e-5
 
 
+@pytest.mark.parametrize("name,n,seed,theta", [("plummer", 9_001, 3, 0.5), ("clustered", 12_000, 4, 0.8),
+                                                ("uniform", 1, 1, 0.5), ("uniform", 37, 2, 0.0)])
+def test_paper_skiplist_variant_parity(NB, oracle, name, n, seed, theta):
+    """Traversal variant 2 (the paper's per-body stackless skip-list DFS,
+    P:222/P:245) against the oracle: counts equal, accelerations in
+    tolerance, and the same lists as the default variant."""
+    pos, vel, mass = generate(name, n, seed)
+    _check_pass(NB, oracle, pos, vel, mass, theta=theta, levels=False, traversal=2)
+    s0 = _run_gpu(NB, pos, vel, mass, theta, 16, traversal=0)
+    s2 = _run_gpu(NB, pos, vel, mass, theta, 16, traversal=2)
+    assert (s0.get_interactions() == s2.get_interactions()).all()
+
+
+def test_paper_skiplist_variant_steps(NB):
+    """Variant 2 inside whole steps (graph capture) matches the default."""
+    pos, vel, mass = generate("disks", 20_000, 11)
+    out = []
+    for v in (0, 2):
+        sim = NB(len(pos), 0.5, EPS, DT, key_bits=16, traversal=v)
+        sim.set_bodies(pos, vel, mass)
+        sim.step(3)
+        out.append((sim.get_positions(), sim.get_interactions()))
+    assert (out[0][1] == out[1][1]).all()
+    assert rel_errors(out[0][0], out[1][0]).max() < 1e-5
+
+
 def test_step_parity_and_determinism(NB, oracle):
     """One full step (force + leapfrog) against the oracle; two GPU runs are
     bit-identical (no float atomics anywhere); graph == plain launches."""
