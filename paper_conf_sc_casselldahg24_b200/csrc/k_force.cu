@@ -560,22 +560,6 @@ __device__ __forceinline__ float warp_maxf(float v) {
   return v;
 }
 
-// a += m r / (|r|^2 + eps^2)^(3/2), r = s - x.  kSoft (eps > 0): r2 > 0 always.
-// kQuad with qid != 0 (warp-uniform): plus node qid's quadrupole [A24].
-template <bool kSoft, bool kQuad>
-__device__ __forceinline__ void interact(Acc& a, const float4& s, float m, const Target& T, const float4* qf,
-                                         uint32_t qid, bool on) {
-  const float dx = s.x - T.x, dy = s.y - T.y, dz = s.z - T.z;
-  const float r2 = fmaf(dz, dz, fmaf(dy, dy, fmaf(dx, dx, T.eps2)));
-  float inv = rsqrt_fast(r2);
-  if (!kSoft) inv = r2 > 0.f ? inv : 0.f;
-  const float w = m * inv * inv * inv;
-  a.x = fmaf(w, dx, a.x);
-  a.y = fmaf(w, dy, a.y);
-  a.z = fmaf(w, dz, a.z);
-  if (kQuad && qid) quad_term(a, dx, dy, dz, inv, qf, qid, on);
-}
-
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 
 // Transposed-phase filter of the fp64 opening test.
@@ -664,8 +648,7 @@ __device__ __forceinline__ void interact2_quad(float2& ax, float2& ay, float2& a
 // Entries [0, cnt) of a pair list; an odd count is padded with a massless
 // entry (it adds exactly 0).
 template <bool kSoft, bool kQuad>
-__device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Target& T, Acc& a, const float4* qf,
-                                           int lane) {
+__device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Target& T, Acc& a, int lane) {
   if constexpr (kQuad) {
     if (nf & 1) {
       if (lane == 0) {
@@ -703,8 +686,7 @@ __device__ __forceinline__ void dense_full(V0Smem<kQuad>& S, int nf, const Targe
 }
 
 template <bool kSoft, bool kQuad>
-__device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane,
-                                           const float4* qf) {
+__device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Target& T, Acc& a, int lane) {
   if constexpr (kQuad) {
     if (np & 1) {
       if (lane == 0) {
@@ -926,7 +908,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       if constexpr (kF64)
         dense_full64<kSoft>(S, nf, T, a);
       else
-        dense_full<kSoft, kQuad>(S, nf, T, a, qf, lane);
+        dense_full<kSoft, kQuad>(S, nf, T, a, lane);
       K6STAT(10, 1);
       K6STAT(11, (nf + 1) >> 1);
       nf = 0;
@@ -935,7 +917,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       if constexpr (kF64)
         dense_part64<kSoft>(S, np, T, a, lane);
       else
-        dense_part<kSoft, kQuad>(S, np, T, a, lane, qf);
+        dense_part<kSoft, kQuad>(S, np, T, a, lane);
       K6STAT(12, 1);
       K6STAT(13, (np + 1) >> 1);
 #ifdef NBODY_K6_STATS
