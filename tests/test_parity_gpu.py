@@ -277,6 +277,33 @@ def test_config3_disks_10M_sampled(NB, oracle):
     _sampled_full_size(NB, oracle, "disks", 10_000_000, 3, 2000)
 
 
+@pytest.mark.slow
+def test_config3_bench_launch_configuration(NB, oracle):
+    """Config 3 at full size in the configuration bench.py times: nbody_step
+    replayed from its CUDA graph on a caller (torch) stream.  The second
+    step's force pass runs on the state left by the first (slot order and
+    all), which is read back with nbody_get_state and given to the oracle;
+    the counts and accelerations of sampled bodies must match it."""
+    import torch
+    n = 10_000_000
+    pos, vel, mass = generate("disks", n, 3)
+    stream = torch.cuda.Stream()
+    sim = NB(n, 0.5, EPS, DT, key_bits=16, stream=stream.cuda_stream)
+    sim.set_bodies(pos, vel, mass)
+    sim.step(1)
+    pm, vi = sim.get_state()              # slot order after step 1
+    ids_state = vi[:, 3].view(np.int32).copy()
+    sim.step(1)                           # its force pass runs on that state
+    acc = sim.get_accel()
+    cnt = sim.get_interactions()
+    targets = np.sort(np.random.default_rng(33).choice(n, 1500, replace=False))
+    ref = oracle.step(pm[:, :3], vi[:, :3], pm[:, 3], ids_state, theta=0.5, eps=EPS, dt=DT, key_bits=16,
+                      integrate=False, targets=targets)
+    ids_t = ref.ids[targets]
+    assert (cnt[ids_t] == ref.count).all()
+    assert_acc_close(acc[ids_t], ref.acc)
+
+
 # ------------------------------------------------------- NEXT-1 all-pairs --
 @pytest.mark.parametrize("name,n,seed,eps", [("plummer", 5000, 60, 1e-3), ("uniform", 3001, 61, 0.0)])
 def test_direct_accel_matches_oracle_direct_sum(NB, oracle, name, n, seed, eps):
