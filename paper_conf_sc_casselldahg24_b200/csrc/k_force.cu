@@ -877,6 +877,10 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     K6STAT(5, __popc(bf));
     K6STAT(6, __popc(bp));
     K6STAT(7, __reduce_add_sync(kFull, part ? __popc(msk) : 0u));
+    K6STAT(32, __reduce_add_sync(kFull, part && __popc(msk) == 1));
+    K6STAT(33, __reduce_add_sync(kFull, part && __popc(msk) == 2));
+    K6STAT(34, __reduce_add_sync(kFull, part && __popc(msk) <= 4));
+    K6STAT(35, __reduce_add_sync(kFull, part && __popc(msk) <= 8));
     K6STAT(8, __popc(bf) * __popc(amask));
 #ifdef NBODY_K6_STATS
     {
