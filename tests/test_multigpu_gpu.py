@@ -289,3 +289,38 @@ def test_peer_exchange_two_processes_ipc(NB, tmp_path):
     for r in range(world):
         assert (np.load(tmp_path / f"x{r}.npy") == ref.get_positions()).all()
         assert (np.load(tmp_path / f"a{r}.npy") == ref.get_accel()).all()
+
+
+@pytest.mark.parametrize("world,balance", [(2, False), (4, True)])
+def test_peer_exchange_with_pipelined_transfers(NB, world, balance):
+    """The bench's N > 1 end-to-end loop: every rank loads its input set with
+    nbody_set_bodies_async, steps, and reads positions with
+    nbody_get_positions_async, two input sets in flight; each rank's outputs
+    equal the single-GPU run's, bit for bit."""
+    import torch
+    n = 20_000
+    sets = [generate("plummer", n, 70 + j) for j in range(2)]
+    kw = {"balance": True} if balance else {}
+    refs = []
+    for pos, vel, mass in sets:
+        ref = NB(n, 0.5, 1e-3, 1e-3, **kw)
+        ref.set_bodies(pos, vel, mass)
+        ref.step(2)
+        refs.append(ref.get_positions())
+    ranks = [NB(n, 0.5, 1e-3, 1e-3, **kw) for _ in range(world)]
+    NB.attach_peers_local(ranks)
+    pinned = [tuple(torch.from_numpy(a).pin_memory() for a in s) for s in sets]
+    outs = [[torch.empty((n, 3), dtype=torch.float32).pin_memory() for _ in sets] for _ in ranks]
+    for j, (hp, hv, hm) in enumerate(pinned):
+        for s in ranks:
+            s.set_bodies_async(hp, hv, hm)
+        for _ in range(2):
+            for s in ranks:
+                s.step(1)
+        for r, s in enumerate(ranks):
+            s.get_positions_async(outs[r][j])
+    for s in ranks:
+        s.sync()
+    for r in range(world):
+        for j in range(len(sets)):
+            assert (outs[r][j].numpy() == refs[j]).all()
