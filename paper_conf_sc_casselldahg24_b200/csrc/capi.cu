@@ -343,8 +343,8 @@ bool balanced(const nbody_ctx* c) { return c->balance && c->xpeer && c->world > 
 nbody_status rank_range(nbody_ctx* c, int q, int64_t* b, int64_t* e) {
   if (!balanced(c)) return nbody_partition(c->n, q, c->world, b, e);
   int64_t r[2];
+  CK(cudaMemcpyAsync(r, c->dpart_used + q, sizeof(r), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
-  CK(cudaMemcpy(r, c->dpart_used + q, sizeof(r), cudaMemcpyDeviceToHost));
   *b = r[0];
   *e = r[1];
   return NBODY_OK;
@@ -414,7 +414,8 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   }
   c->last_sorted = resort;
   int x_kernels = 0;
-  if (c->xpeer && integrate) {  // every rank has consumed the old state: peers may overwrite it
+  if (c->xpeer) {  // every rank has consumed the old state: peers may overwrite it (and, for a
+                   // force-only pass, no peer still reads the acc/cnt/gcost this pass rewrites)
     launch_xbarrier(c->peers, c->xepoch, 0, c->xerr, s);
     ++x_kernels;
   }
@@ -547,7 +548,7 @@ nbody_status sync_stream(nbody_ctx* c) {
 
 // Fill the peer table from every rank's arena base (layouts are identical:
 // same N, same plan) and switch the context to the fused exchange.
-void attach_peer_bases(nbody_ctx* c, char* const* base, int rank, int world) {
+nbody_status attach_peer_bases(nbody_ctx* c, char* const* base, int rank, int world) {
   auto at = [&](int q, const void* own) { return base[q] + (static_cast<const char*>(own) - c->arena); };
   PeerTable& pt = c->peers;
   pt.G = world;
@@ -565,9 +566,11 @@ void attach_peer_bases(nbody_ctx* c, char* const* base, int rank, int world) {
   // NEXT-3(i): the first pass uses the equal slices [A21]
   int64_t bounds[kMaxPeers + 1];
   for (int q = 0; q <= world; ++q) bounds[q] = std::min(c->n, int64_t(q) * c->own_s);
-  cudaMemcpy(c->dpart, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice);
-  cudaMemcpy(c->dpart_used, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice);
+  CK(cudaMemcpyAsync(c->dpart, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(c->dpart_used, bounds, sizeof(int64_t) * (world + 1), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
   drop_graph(c);
+  return NBODY_OK;
 }
 
 struct PeerDesc {  // nbody_peer_handle's 128-byte record
@@ -575,6 +578,7 @@ struct PeerDesc {  // nbody_peer_handle's 128-byte record
   int64_t n;
   uint64_t arena_bytes;
   uint32_t magic;
+  char pci[20];  // the owner's device, as a PCI bus id (device ordinals differ between processes)
 };
 static_assert(sizeof(PeerDesc) <= 128, "peer descriptor must fit in 128 bytes");
 constexpr uint32_t kPeerMagic = 0x4e42584bu;
@@ -758,17 +762,19 @@ nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, 
   const int64_t n = c->n;
   const float *dp = pos, *dv = vel, *dm = mass;
   cudaStream_t s = c->stream;
+  // host inputs are staged in buffers only this rank reads (peers read acc
+  // and cnt directly in the peer-exchange mode)
   if (!is_device_ptr(pos)) {
-    CK(cudaMemcpyAsync(c->acc, pos, 12 * size_t(n), cudaMemcpyDefault, s));
-    dp = reinterpret_cast<const float*>(c->acc);
+    CK(cudaMemcpyAsync(c->stage, pos, 12 * size_t(n), cudaMemcpyDefault, s));
+    dp = reinterpret_cast<const float*>(c->stage);
   }
   if (!is_device_ptr(vel)) {
-    CK(cudaMemcpyAsync(c->stage, vel, 12 * size_t(n), cudaMemcpyDefault, s));
-    dv = reinterpret_cast<const float*>(c->stage);
+    CK(cudaMemcpyAsync(c->out3, vel, 12 * size_t(n), cudaMemcpyDefault, s));
+    dv = c->out3;
   }
   if (!is_device_ptr(mass)) {
-    CK(cudaMemcpyAsync(c->cnt, mass, 4 * size_t(n), cudaMemcpyDefault, s));
-    dm = reinterpret_cast<const float*>(c->cnt);
+    CK(cudaMemcpyAsync(c->stage2, mass, 4 * size_t(n), cudaMemcpyDefault, s));
+    dm = reinterpret_cast<const float*>(c->stage2);
   }
   CK(cudaMemsetAsync(c->bad, 0, sizeof(int), s));
   launch_pack_bodies(dp, dv, dm, n, c->pm[0], c->vi[0], c->bad, s);
@@ -1198,6 +1204,7 @@ nbody_status nbody_peer_handle(nbody_ctx* c, void* out) {
   d.n = c->n;
   d.arena_bytes = c->arena_bytes;
   d.magic = kPeerMagic;
+  CK(cudaDeviceGetPCIBusId(d.pci, sizeof(d.pci), c->device));
   std::memset(out, 0, 128);
   std::memcpy(out, &d, sizeof(d));
   return NBODY_OK;
@@ -1229,19 +1236,42 @@ nbody_status nbody_attach_peers(nbody_ctx* c, const void* handles, int rank, int
       base[q] = c->arena;
       continue;
     }
+    auto unmap = [&]() {
+      for (int k = 0; k < q; ++k)
+        if (c->peer_map[k]) cudaIpcCloseMemHandle(c->peer_map[k]), c->peer_map[k] = nullptr;
+    };
+    // the peer's arena must be reachable by loads/stores from this device
+    // (NVLink/NVSwitch or PCIe P2P); say so instead of faulting in K7
+    d.pci[sizeof(d.pci) - 1] = 0;
+    int pdev = -1;
+    if (cudaDeviceGetByPCIBusId(&pdev, d.pci) != cudaSuccess) {
+      cudaGetLastError();
+      unmap();
+      return fail(c, NBODY_EINVAL, "peer " + std::to_string(q) + ": device " + d.pci +
+                                       " is not visible to this process (CUDA_VISIBLE_DEVICES must expose every "
+                                       "rank's GPU for the peer exchange; use the NCCL exchange otherwise)");
+    }
+    if (pdev != c->device) {
+      int ok = 0;
+      CK(cudaDeviceCanAccessPeer(&ok, c->device, pdev));
+      if (!ok) {
+        unmap();
+        return fail(c, NBODY_EINVAL, "peer " + std::to_string(q) + ": no peer access from device " +
+                                         std::to_string(c->device) + " to device " + std::to_string(pdev) +
+                                         " (use the NCCL exchange)");
+      }
+    }
     void* p = nullptr;
     const cudaError_t e = cudaIpcOpenMemHandle(&p, d.ipc, cudaIpcMemLazyEnablePeerAccess);
     if (e != cudaSuccess) {
       cudaGetLastError();
-      for (int k = 0; k < q; ++k)
-        if (c->peer_map[k]) cudaIpcCloseMemHandle(c->peer_map[k]), c->peer_map[k] = nullptr;
+      unmap();
       return fail(c, NBODY_ECUDA, "cudaIpcOpenMemHandle(peer " + std::to_string(q) + "): " + cudaGetErrorString(e));
     }
     c->peer_map[q] = p;
     base[q] = static_cast<char*>(p);
   }
-  attach_peer_bases(c, base, rank, world);
-  return NBODY_OK;
+  return attach_peer_bases(c, base, rank, world);
 }
 
 nbody_status nbody_attach_peers_local(nbody_ctx** ctxs, int world) {
@@ -1268,7 +1298,10 @@ nbody_status nbody_attach_peers_local(nbody_ctx** ctxs, int world) {
     }
   char* base[kMaxPeers] = {};
   for (int q = 0; q < world; ++q) base[q] = ctxs[q]->arena;
-  for (int r = 0; r < world; ++r) attach_peer_bases(ctxs[r], base, r, world);
+  for (int r = 0; r < world; ++r) {
+    const nbody_status st = attach_peer_bases(ctxs[r], base, r, world);
+    if (st != NBODY_OK) return st;
+  }
   return NBODY_OK;
 }
 

@@ -415,6 +415,9 @@ __global__ __launch_bounds__(kV2Threads) void k_force_skiplist(const ForceParams
   const int64_t k0 = tb + int64_t(blockIdx.x) * kV2Threads + (threadIdx.x & ~31);
   const int64_t k = k0 + lane;
   const bool active = k < te;
+  // idle warps past the range end store nothing (their gcost entry belongs
+  // to the next rank, or lies past the last group)
+  if (__ballot_sync(kFull, active) == 0) return;
   const Target T = load_target(P, k, active);
   const Walk W = make_walk(P);
   const uint32_t kid = W.leaf0 + uint32_t(k);
@@ -462,7 +465,10 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_V0_MINB
 #define NBODY_V0_MINB 8
 #endif
-constexpr int kCapA = 128;          // box-phase stack (ids)
+#ifndef NBODY_CAP_A
+#define NBODY_CAP_A 128
+#endif
+constexpr int kCapA = NBODY_CAP_A;  // box-phase stack (ids)
 constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 #ifndef NBODY_CAP_F
 #define NBODY_CAP_F 96
@@ -1108,6 +1114,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
             two = ((2u * g + 1u) << (l - 1)) - leaf0 < n;
           } else {
             cls = 3;
+            K6STAT(36, dmax2 * (1.f + 4e-6f) < c.x);  // an all-open node handed to T by the capacity guard
           }
         }
       }
