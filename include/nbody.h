@@ -145,6 +145,36 @@ nbody_status nbody_select_device(int device);
  *   sizes are fixed by N).  *out is set to NULL on failure. */
 nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx **out);
 
+/* ---- caller-owned device memory (PyTorch as the allocator) -------------
+ * Tree and buffer sizes follow from N alone ("the size of the tree
+ * is predetermined by the number of bodies"), so the whole device footprint
+ * of a context is known before it exists.  nbody_workspace_bytes returns the
+ * bytes of the base workspace (state, keys, sort scratch, tree records,
+ * exchange flags) for n bodies on the CURRENT device (the layout depends on
+ * its SM count); one layout serves every world <= 256 and every key width
+ * b <= 21, so `world` and `key_bits` are only range-checked (0 on a bad
+ * argument).  nbody_workspace_bytes_ex adds the optional buffers a context
+ * allocates on first use: NBODY_WS_QUAD (quadrupole moments, 80 B per
+ * internal node), NBODY_WS_XFER (pipelined-transfer staging, 80 B per body),
+ * NBODY_WS_FP64 (the FP64 mode's state and tree). */
+enum { NBODY_WS_QUAD = 1, NBODY_WS_XFER = 2, NBODY_WS_FP64 = 4 };
+size_t nbody_workspace_bytes(int64_t n, int world, int key_bits);
+size_t nbody_workspace_bytes_ex(int64_t n, int world, int key_bits, unsigned features);
+/* As nbody_create, but every device buffer of the context is carved, in a
+ * fixed order, from dev_workspace[bytes] (a device pointer on the current
+ * device, 256-byte aligned, e.g. a torch.empty(bytes, dtype=torch.uint8,
+ * device="cuda") tensor): the library allocates no device memory for the
+ * context's state.  The caller owns the workspace and must keep it alive
+ * until nbody_destroy.  bytes >= nbody_workspace_bytes(n, ...) or
+ * NBODY_ENOMEM; optional buffers are taken from the rest of the workspace
+ * when first used, and NBODY_ENOMEM is returned then if it does not cover
+ * them (size it with nbody_workspace_bytes_ex).  NBODY_EINVAL for a null,
+ * misaligned, host or other-device pointer.  Results are bit-identical to
+ * a context made by nbody_create.  (nbody_direct_accel, a sampling tool,
+ * still takes stream-ordered scratch from the CUDA runtime.) */
+nbody_status nbody_create_ws(int64_t n, double theta, double eps, double dt, void *dev_workspace, size_t bytes,
+                             nbody_ctx **out);
+
 /* Set an option (see enum).  Returns NBODY_EINVAL for an unknown option or
  * value, NBODY_ESTATE if the option can no longer change. */
 nbody_status nbody_set_option(nbody_ctx *ctx, int option, int64_t value);
@@ -223,6 +253,19 @@ nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
  * accuracy against the exact field (config 5). */
 nbody_status nbody_direct_accel(nbody_ctx *ctx, const int64_t *ids, int64_t nt, double *out);
 
+/* ---- NEXT-1: the All-Pairs baseline in fp32 at full N ---
+ * Softened direct sum of Eq. 1 [A1] at the current positions for the
+ * bodies with ids[nt] against ALL n sources, in the fp32 arithmetic of the
+ * force kernel's interactions (fp32 differences, FMA, MUFU rsqrt; the
+ * target itself adds 0), fp32 partial sums per 2048-source tile and fp64
+ * across tiles; out[nt][3] fp64 (host or device).  ids host or device
+ * (host ids are range-checked).  Deterministic.  If kernel_ms is not NULL
+ * it receives the device time of the all-pairs kernel alone (CUDA events
+ * on the context stream) -- the calibration of the FP32 interaction rate
+ * the Barnes-Hut force kernel is measured against.  Takes stream-ordered
+ * scratch of about 32 B x nt x (source chunks) from the CUDA runtime. */
+nbody_status nbody_allpairs_accel(nbody_ctx *ctx, const int64_t *ids, int64_t nt, double *out, float *kernel_ms);
+
 /* ---- multi-GPU: Hilbert-range partition ------------------
  * Every rank holds the whole body state and builds the same tree (all stages
  * up to the tree are deterministic, so the replicas are bit-identical); rank
@@ -247,6 +290,18 @@ nbody_status nbody_nccl_unique_id(void *out128);
 /* Create an NCCL communicator for (rank, world) on the current device and
  * partition the context accordingly.  Collective; call before stepping. */
 nbody_status nbody_attach_nccl(nbody_ctx *ctx, const void *unique_id128, int rank, int world);
+/* Use an existing NCCL communicator (ncclComm_t passed as void*), e.g. the
+ * one torch.distributed's ProcessGroupNCCL created for this device
+ * (ProcessGroupNCCL._comm_ptr(), after eager initialisation with device_id):
+ * the exchange runs on it instead of a communicator of the library's own.
+ * rank and world must equal the communicator's (NBODY_EINVAL otherwise, or
+ * if it belongs to another device).  The caller keeps ownership: the
+ * communicator must outlive the context and is not destroyed by
+ * nbody_destroy.  The library must be linked against the same NCCL as the
+ * communicator's creator (build.py links the NCCL that the torch wheel
+ * ships).  NBODY_ESTATE if a communicator or peers are already attached;
+ * NBODY_ENCCL if the library was built without NCCL. */
+nbody_status nbody_attach_comm(nbody_ctx *ctx, void *nccl_comm, int rank, int world);
 /* Partition without a communicator (1 <= world <= 256). */
 nbody_status nbody_set_partition(nbody_ctx *ctx, int rank, int world);
 /* The context's rank, world and owned sorted-slot range [begin, end). */

@@ -29,6 +29,10 @@ NBODY_OPT_MULTIPOLE = 8
 NBODY_OPT_BALANCE = 9
 NBODY_OPT_PRECISION = 10
 
+NBODY_WS_QUAD = 1
+NBODY_WS_XFER = 2
+NBODY_WS_FP64 = 4
+
 _STATUS = {0: "NBODY_OK", -1: "NBODY_EINVAL", -2: "NBODY_ENOMEM", -3: "NBODY_ECUDA", -4: "NBODY_ENCCL",
            -5: "NBODY_ESTATE"}
 
@@ -56,6 +60,11 @@ SIGNATURES = {
     "nbody_select_device": (_S, [C.c_int]),
     "nbody_debug_force_stats": (C.c_int, [_P, C.c_int]),
     "nbody_create": (_S, [_I64, C.c_double, C.c_double, C.c_double, C.POINTER(_P)]),
+    "nbody_create_ws": (_S, [_I64, C.c_double, C.c_double, C.c_double, _P, C.c_size_t, C.POINTER(_P)]),
+    "nbody_workspace_bytes": (C.c_size_t, [_I64, C.c_int, C.c_int]),
+    "nbody_workspace_bytes_ex": (C.c_size_t, [_I64, C.c_int, C.c_int, C.c_uint]),
+    "nbody_attach_comm": (_S, [_P, _P, C.c_int, C.c_int]),
+    "nbody_allpairs_accel": (_S, [_P, _P, _I64, _P, _P]),
     "nbody_set_option": (_S, [_P, C.c_int, _I64]),
     "nbody_set_bodies": (_S, [_P, _P, _P, _P]),
     "nbody_set_bodies_async": (_S, [_P, _P, _P, _P]),

@@ -74,6 +74,12 @@ struct nbody_ctx {
   int sort_every = 1;                   // re-sort every k-th step
   bool last_sorted = false;
   void* quad_arena = nullptr;           // NEXT-4 S64 + qf (lazy)
+  // caller-owned workspace (nbody_create_ws): every device buffer of the
+  // context is carved from it in a fixed order; the library then allocates
+  // no device memory of its own for the context's state
+  bool ws_ext = false;
+  char* ws = nullptr;
+  size_t ws_bytes = 0, ws_used = 0;
 
   // partition over ranks [A21]: rank r owns sorted slots [own_b, own_e),
   // own_s = slice length (a multiple of 32 so warp groups match 1 GPU)
@@ -81,6 +87,7 @@ struct nbody_ctx {
   int64_t own_s = 0, own_b = 0, own_e = 0;
 #ifdef NBODY_WITH_NCCL
   ncclComm_t comm = nullptr;
+  bool comm_borrowed = false;  // nbody_attach_comm: the caller's communicator, not destroyed here
 #endif
   // fused K7 + exchange over peer memory (k_exchange.cu)
   size_t arena_bytes = 0;
@@ -201,13 +208,16 @@ int64_t plan_tree(TreeView& t, int64_t n) {
   return int64_t(2) << t.L;
 }
 
-nbody_status allocate(nbody_ctx* c) {
-  const int64_t n = c->n;
-  const int64_t ids = plan_tree(c->tree, n);   // rec / s2f cover leaves too
+// Sizes of the base arena's buffers, in carving order (sz[32]); returns the
+// count.  Depends on N (tree sizes are fixed by N) and the SM count
+// (bbox partials) only: every key width (b <= 21) and every world <= 256
+// fit the same layout.
+int arena_plan(int64_t n, int nsm, size_t* sz) {
+  TreeView t{};
+  const int64_t ids = plan_tree(t, n);         // rec / s2f cover leaves too
   const int64_t inner = ids / 2;                // pred / mom / box: internal ids < 2^L
-  c->nbbox = 2 * c->nsm;
+  const int nbbox = 2 * nsm;
   const int64_t tiles = sort_tiles(n);
-  size_t sz[32];
   int k = 0;
   sz[k++] = 16 * size_t(n + kPartPad);              // pm0 (room for G * S records)
   sz[k++] = 16 * size_t(n + kPartPad);              // vi0
@@ -222,7 +232,7 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 16 * size_t(n + kPartPad);              // stage (gathered acc for G > 1)
   sz[k++] = 4 * size_t(n + kPartPad);               // stage2 (gathered counts)
   sz[k++] = 12 * size_t(n);                         // out3 (by-id outputs for host callers)
-  sz[k++] = sizeof(float) * 6 * size_t(c->nbbox);   // bbox partials
+  sz[k++] = sizeof(float) * 6 * size_t(nbbox);   // bbox partials
   sz[k++] = sizeof(GridInfo);
   sz[k++] = 8;                                      // total
   sz[k++] = 8;                                      // bad
@@ -236,13 +246,86 @@ nbody_status allocate(nbody_ctx* c) {
   sz[k++] = 16 * size_t(inner);                     // tf
   sz[k++] = 4 * size_t(n / 32 + 1);                 // gcost
   sz[k++] = 512;                                    // exchange flags, epochs, error, partitions
+  return k;
+}
+
+size_t sum_aligned(const size_t* sz, int k) {
   size_t total = 0;
   for (int i = 0; i < k; ++i) total += align_up(sz[i]);
-  cudaError_t e = cudaMalloc(&c->arena, total);
+  return total;
+}
+
+size_t arena_bytes_for(int64_t n, int nsm) {
+  size_t sz[32];
+  return sum_aligned(sz, arena_plan(n, nsm, sz));
+}
+
+// Optional buffers, allocated on first use (NBODY_WS_* in nbody.h).
+size_t quad_bytes_for(int64_t n) {
+  TreeView t{};
+  const size_t inner = size_t(plan_tree(t, n) / 2);
+  return align_up(48 * inner + 32 * inner);
+}
+size_t xfer_bytes_for(int64_t n) { return align_up(align_up(2 * 28 * size_t(n)) + align_up(2 * 12 * size_t(n)) + 256); }
+size_t f64_plan(int64_t n, int nsm, size_t* sz) {
+  TreeView t{};
+  const size_t ids = size_t(plan_tree(t, n)), inner = ids / 2;
+  const int nbbox = 2 * nsm;
+  int k = 0;
+  sz[k++] = 32 * size_t(n);              // pm64[0]
+  sz[k++] = 32 * size_t(n);              // vi64[0]
+  sz[k++] = 32 * size_t(n);              // vi64[1]
+  sz[k++] = 32 * ids;                    // rec64 (leaf ids = pm64[1])
+  sz[k++] = 32 * inner;                  // blo64
+  sz[k++] = 32 * inner;                  // bhi64
+  sz[k++] = 32 * size_t(n);              // acc64
+  sz[k++] = 48 * size_t(nbbox) + 24 * size_t(n);  // bbox partials + staging
+  return size_t(k);
+}
+size_t f64_bytes_for(int64_t n, int nsm) {
+  size_t sz[8];
+  return sum_aligned(sz, int(f64_plan(n, nsm, sz)));
+}
+
+// Device memory for the context: from the caller's workspace (create_ws),
+// else cudaMalloc.  `what` names the buffer in the error.
+nbody_status dev_alloc(nbody_ctx* c, size_t bytes, void** out, const char* what) {
+  *out = nullptr;
+  bytes = align_up(bytes);
+  if (c->ws_ext) {
+    if (c->ws_used + bytes > c->ws_bytes)
+      return fail(c, NBODY_ENOMEM, std::string(what) + ": the caller's workspace is too small (" +
+                                       std::to_string(c->ws_bytes) + " bytes; nbody_workspace_bytes_ex gives the size "
+                                       "with the optional buffers)");
+    *out = c->ws + c->ws_used;
+    c->ws_used += bytes;
+    return NBODY_OK;
+  }
+  const cudaError_t e = cudaMalloc(out, bytes);
   if (e != cudaSuccess) {
     cudaGetLastError();
-    c->arena = nullptr;
-    return fail(c, NBODY_ENOMEM, "cudaMalloc of " + std::to_string(total) + " bytes failed");
+    *out = nullptr;
+    return fail(c, NBODY_ENOMEM, std::string(what) + ": cudaMalloc of " + std::to_string(bytes) + " bytes failed");
+  }
+  return NBODY_OK;
+}
+void dev_free(nbody_ctx* c, void* p) {
+  if (p && !c->ws_ext) cudaFree(p);
+}
+
+nbody_status allocate(nbody_ctx* c) {
+  const int64_t n = c->n;
+  plan_tree(c->tree, n);
+  c->nbbox = 2 * c->nsm;
+  const int64_t tiles = sort_tiles(n);
+  size_t sz[32];
+  const int k = arena_plan(n, c->nsm, sz);
+  const size_t total = sum_aligned(sz, k);
+  {
+    void* a = nullptr;
+    const nbody_status st = dev_alloc(c, total, &a, "state and tree arena");
+    if (st != NBODY_OK) return st;
+    c->arena = static_cast<char*>(a);
   }
   char* p = c->arena;
   int i = 0;
@@ -286,7 +369,7 @@ nbody_status allocate(nbody_ctx* c) {
   // leaves always interact when reached: thresholds (-inf, -inf), set once
   const float ninf = -INFINITY;
   launch_fill_float2(c->tree.rc + (int64_t(1) << c->tree.L), n, make_float2(ninf, ninf), nullptr);
-  e = cudaMemset(c->xflags, 0, 512);
+  cudaError_t e = cudaMemset(c->xflags, 0, 512);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
   c->sort.n = n;
@@ -300,24 +383,11 @@ nbody_status allocate(nbody_ctx* c) {
 // NEXT-2 FP64 mode buffers (one allocation, on first use).
 nbody_status alloc_f64(nbody_ctx* c) {
   const int64_t n = c->n;
-  const size_t ids = size_t(1) << (c->tree.L + 1), inner = ids / 2;
   size_t sz[8];
-  int k = 0;
-  sz[k++] = 32 * size_t(n);              // pm64[0]
-  sz[k++] = 32 * size_t(n);              // vi64[0]
-  sz[k++] = 32 * size_t(n);              // vi64[1]
-  sz[k++] = 32 * ids;                    // rec64 (leaf ids = pm64[1])
-  sz[k++] = 32 * inner;                  // blo64
-  sz[k++] = 32 * inner;                  // bhi64
-  sz[k++] = 32 * size_t(n);              // acc64
-  sz[k++] = 48 * size_t(c->nbbox) + 24 * size_t(n);  // bbox partials + staging
-  size_t total = 0;
-  for (int i = 0; i < k; ++i) total += align_up(sz[i]);
-  cudaError_t e = cudaMalloc(&c->arena64, total);
-  if (e != cudaSuccess) {
-    cudaGetLastError();
-    c->arena64 = nullptr;
-    return fail(c, NBODY_ENOMEM, "FP64 mode buffers (" + std::to_string(total) + " bytes)");
+  f64_plan(n, c->nsm, sz);
+  {
+    const nbody_status st = dev_alloc(c, sum_aligned(sz, 8), &c->arena64, "FP64 mode buffers");
+    if (st != NBODY_OK) return st;
   }
   char* p = static_cast<char*>(c->arena64);
   int i = 0;
@@ -578,8 +648,34 @@ struct PeerDesc {  // nbody_peer_handle's 128-byte record
   int64_t n;
   uint64_t arena_bytes;
   uint32_t magic;
-  char pci[20];  // the owner's device, as a PCI bus id (device ordinals differ between processes)
+  char pci[20];     // the owner's device, as a PCI bus id (device ordinals differ between processes)
+  uint64_t offset;  // the arena's offset in the allocation the IPC handle maps (a caller workspace,
+                    // e.g. a torch tensor, may sit inside a larger cudaMalloc block)
 };
+
+// Base address of the device allocation containing p (driver API
+// cuMemGetAddressRange, reached through the runtime's entry-point query so
+// the library needs no libcuda link).
+nbody_status alloc_base(nbody_ctx* c, const void* p, const char** base) {
+  using Fn = int (*)(unsigned long long*, size_t*, unsigned long long);
+  static Fn fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuMemGetAddressRange", &f, 12000, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !f) {
+      cudaGetLastError();
+      return fail(c, NBODY_ECUDA, "cuMemGetAddressRange is not available");
+    }
+    fn = reinterpret_cast<Fn>(f);
+  }
+  unsigned long long b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, reinterpret_cast<unsigned long long>(p)) != 0)
+    return fail(c, NBODY_ECUDA, "cuMemGetAddressRange failed for the arena");
+  *base = reinterpret_cast<const char*>(b);
+  return NBODY_OK;
+}
 static_assert(sizeof(PeerDesc) <= 128, "peer descriptor must fit in 128 bytes");
 constexpr uint32_t kPeerMagic = 0x4e42584bu;
 
@@ -599,11 +695,13 @@ nbody_status nbody_select_device(int device) {
   return cudaSetDevice(device) == cudaSuccess ? NBODY_OK : NBODY_ECUDA;
 }
 
-nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx** out) {
+static nbody_status create_impl(int64_t n, double theta, double eps, double dt, void* ws, size_t ws_bytes,
+                                nbody_ctx** out) {
   if (!out) return NBODY_EINVAL;
   *out = nullptr;
   if (n < 1 || n >= (int64_t(1) << 30)) return NBODY_EINVAL;
   if (!std::isfinite(theta) || theta < 0 || !std::isfinite(eps) || eps < 0 || !std::isfinite(dt)) return NBODY_EINVAL;
+  if (ws && (reinterpret_cast<uintptr_t>(ws) & 255u)) return NBODY_EINVAL;  // 256-byte aligned (torch: 512)
   nbody_ctx* c = new (std::nothrow) nbody_ctx;
   if (!c) return NBODY_ENOMEM;
   c->n = n;
@@ -617,6 +715,18 @@ nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_
   if (cudaGetDevice(&c->device) != cudaSuccess) return bail(NBODY_ECUDA);
   cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device);
   if (c->nsm <= 0) c->nsm = kNumSMs;
+  if (ws) {
+    if (!is_device_ptr(ws)) return bail(NBODY_EINVAL);
+    cudaPointerAttributes pa;
+    if (cudaPointerGetAttributes(&pa, ws) != cudaSuccess || pa.device != c->device) {
+      cudaGetLastError();
+      return bail(NBODY_EINVAL);  // the workspace must live on the current device
+    }
+    if (ws_bytes < arena_bytes_for(n, c->nsm)) return bail(NBODY_ENOMEM);
+    c->ws_ext = true;
+    c->ws = static_cast<char*>(ws);
+    c->ws_bytes = ws_bytes;
+  }
   if (cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking) != cudaSuccess) return bail(NBODY_ECUDA);
   if (cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking) != cudaSuccess) return bail(NBODY_ECUDA);
   for (auto& e : c->ev)
@@ -631,6 +741,43 @@ nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_
   c->sort.passes = (3 * c->b + 7) / 8;
   *out = c;
   return NBODY_OK;
+}
+
+nbody_status nbody_create(int64_t n, double theta, double eps, double dt, nbody_ctx** out) {
+  return create_impl(n, theta, eps, dt, nullptr, 0, out);
+}
+
+nbody_status nbody_create_ws(int64_t n, double theta, double eps, double dt, void* dev_workspace, size_t bytes,
+                             nbody_ctx** out) {
+  if (!dev_workspace) {
+    if (out) *out = nullptr;
+    return NBODY_EINVAL;
+  }
+  return create_impl(n, theta, eps, dt, dev_workspace, bytes, out);
+}
+
+static int current_sms() {
+  int dev = 0, nsm = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+    cudaGetLastError();
+    nsm = kNumSMs;
+  }
+  return nsm > 0 ? nsm : kNumSMs;
+}
+
+size_t nbody_workspace_bytes_ex(int64_t n, int world, int key_bits, unsigned features) {
+  if (n < 1 || n >= (int64_t(1) << 30) || world < 1 || world > kMaxWorld || key_bits < 0 || key_bits > 21) return 0;
+  if (features & ~unsigned(NBODY_WS_QUAD | NBODY_WS_XFER | NBODY_WS_FP64)) return 0;
+  const int nsm = current_sms();
+  size_t total = arena_bytes_for(n, nsm);  // one layout for every world <= 256 and b <= 21
+  if (features & NBODY_WS_QUAD) total += quad_bytes_for(n);
+  if (features & NBODY_WS_XFER) total += xfer_bytes_for(n);
+  if (features & NBODY_WS_FP64) total += align_up(f64_bytes_for(n, nsm));
+  return total;
+}
+
+size_t nbody_workspace_bytes(int64_t n, int world, int key_bits) {
+  return nbody_workspace_bytes_ex(n, world, key_bits, 0u);
 }
 
 nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
@@ -663,12 +810,8 @@ nbody_status nbody_set_option(nbody_ctx* c, int option, int64_t value) {
       if (value == 2 && c->traversal == 2) return fail(c, NBODY_EINVAL, "traversal variant 2 is monopole only");
       if (value == 2 && !c->tree.S64) {  // allocated on first use: 80 B per internal id
         const size_t inner = size_t(1) << c->tree.L;
-        cudaError_t e = cudaMalloc(&c->quad_arena, 48 * inner + 32 * inner);
-        if (e != cudaSuccess) {
-          cudaGetLastError();
-          c->quad_arena = nullptr;
-          return fail(c, NBODY_ENOMEM, "quadrupole arrays");
-        }
+        const nbody_status st = dev_alloc(c, quad_bytes_for(c->n), &c->quad_arena, "quadrupole arrays");
+        if (st != NBODY_OK) return st;
         c->tree.S64 = reinterpret_cast<Quad64*>(c->quad_arena);
         c->tree.qf = reinterpret_cast<float4*>(static_cast<char*>(c->quad_arena) + 48 * inner);
       }
@@ -804,11 +947,8 @@ static nbody_status ensure_xfer(nbody_ctx* c) {
     for (cudaEvent_t* e : {&c->ev_in_copied[k], &c->ev_in_used[k], &c->ev_out_ready[k], &c->ev_out_copied[k]})
       if (!*e) CK(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
   void* p = nullptr;
-  const cudaError_t e = cudaMalloc(&p, align_up(2 * 28 * n) + align_up(2 * 12 * n) + 256);
-  if (e != cudaSuccess) {
-    cudaGetLastError();
-    return fail(c, NBODY_ENOMEM, "staging buffers of the pipelined transfers");
-  }
+  const nbody_status st = dev_alloc(c, xfer_bytes_for(c->n), &p, "staging buffers of the pipelined transfers");
+  if (st != NBODY_OK) return st;
   c->xfer = static_cast<char*>(p);
   c->bad_async = reinterpret_cast<int*>(c->xfer + align_up(2 * 28 * n) + align_up(2 * 12 * n));
   CK(cudaMemsetAsync(c->bad_async, 0, sizeof(int), c->stream));
@@ -1099,6 +1239,44 @@ nbody_status nbody_direct_accel(nbody_ctx* c, const int64_t* ids, int64_t nt, do
   return sync_stream(c);
 }
 
+nbody_status nbody_allpairs_accel(nbody_ctx* c, const int64_t* ids, int64_t nt, double* out, float* kernel_ms) {
+  CHECK_CTX(c);
+  if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
+  if (nt < 0 || (nt > 0 && (!ids || !out))) return fail(c, NBODY_EINVAL, "bad target list");
+  if (c->f64) return fail(c, NBODY_EINVAL, "nbody_allpairs_accel works on the fp32 state (precision 32)");
+  if (kernel_ms) *kernel_ms = 0.f;
+  if (nt == 0) return NBODY_OK;
+  const bool ids_dev = is_device_ptr(ids);
+  if (!ids_dev)
+    for (int64_t i = 0; i < nt; ++i)
+      if (ids[i] < 0 || ids[i] >= c->n) return fail(c, NBODY_EINVAL, "id out of range");
+  const int64_t chunks = allpairs_chunks(c->n, nt, c->nsm);
+  cudaStream_t s = c->stream;
+  char* tmp = nullptr;
+  const size_t bi = align_up(8 * size_t(nt)), bt = align_up(4 * size_t(nt)), bp = align_up(32 * size_t(chunks * nt));
+  const size_t bo = align_up(24 * size_t(nt));
+  CK(cudaMallocAsync(reinterpret_cast<void**>(&tmp), bi + bt + bp + bo, s));
+  int64_t* d_ids = reinterpret_cast<int64_t*>(tmp);
+  uint32_t* d_tslot = reinterpret_cast<uint32_t*>(tmp + bi);
+  double4* d_part = reinterpret_cast<double4*>(tmp + bi + bt);
+  double* d_out = reinterpret_cast<double*>(tmp + bi + bt + bp);
+  cudaError_t e = cudaMemcpyAsync(d_ids, ids, 8 * size_t(nt), cudaMemcpyDefault, s);
+  if (e == cudaSuccess) {
+    launch_target_slots(c->vi[0], c->n, d_ids, nt, c->stage2, d_tslot, s);
+    launch_allpairs32(c->pm[0], c->n, d_tslot, nt, float(c->eps * c->eps), chunks, d_part, d_out,
+                      kernel_ms ? c->ev[0] : nullptr, kernel_ms ? c->ev[1] : nullptr, s);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaMemcpyAsync(out, d_out, 24 * size_t(nt), cudaMemcpyDefault, s);
+  cudaFreeAsync(tmp, s);
+  if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
+  const nbody_status st = sync_stream(c);
+  if (st != NBODY_OK) return st;
+  if (kernel_ms) CK(cudaEventElapsedTime(kernel_ms, c->ev[0], c->ev[1]));
+  c->ev_valid = false;  // the stage events now hold the all-pairs kernel
+  return NBODY_OK;
+}
+
 // ---- partition / multi-GPU -------------------------------------------------
 
 nbody_status nbody_set_partition(nbody_ctx* c, int rank, int world) {
@@ -1194,13 +1372,44 @@ nbody_status nbody_attach_nccl(nbody_ctx* c, const void* unique_id, int rank, in
 #endif
 }
 
+nbody_status nbody_attach_comm(nbody_ctx* c, void* nccl_comm, int rank, int world) {
+  CHECK_CTX(c);
+  if (!nccl_comm || world < 1 || world > kMaxWorld || rank < 0 || rank >= world)
+    return fail(c, NBODY_EINVAL, "need a communicator and 0 <= rank < world <= 256");
+  if (c->f64) return fail(c, NBODY_EINVAL, "the FP64 mode runs on a single rank");
+#ifdef NBODY_WITH_NCCL
+  if (c->comm) return fail(c, NBODY_ESTATE, "a communicator is already attached");
+  if (c->xpeer) return fail(c, NBODY_ESTATE, "peers are attached");
+  ncclComm_t comm = static_cast<ncclComm_t>(nccl_comm);
+  int r = -1, w = -1, d = -1;
+  ncclResult_t e = ncclCommUserRank(comm, &r);
+  if (e == ncclSuccess) e = ncclCommCount(comm, &w);
+  if (e == ncclSuccess) e = ncclCommCuDevice(comm, &d);
+  if (e != ncclSuccess) return fail(c, NBODY_ENCCL, std::string("communicator query: ") + ncclGetErrorString(e));
+  if (r != rank || w != world)
+    return fail(c, NBODY_EINVAL, "the communicator is rank " + std::to_string(r) + " of " + std::to_string(w));
+  if (d != c->device) return fail(c, NBODY_EINVAL, "the communicator belongs to another device");
+  c->comm = comm;
+  c->comm_borrowed = true;
+  set_part(c, rank, world);
+  drop_graph(c);
+  return NBODY_OK;
+#else
+  return fail(c, NBODY_ENCCL, "library built without NCCL");
+#endif
+}
+
 // ---- fused exchange over peer memory --------------------------------------
 
 nbody_status nbody_peer_handle(nbody_ctx* c, void* out) {
   CHECK_CTX(c);
   if (!out) return fail(c, NBODY_EINVAL, "null output");
   PeerDesc d{};
-  CK(cudaIpcGetMemHandle(&d.ipc, c->arena));
+  const char* base = nullptr;
+  const nbody_status st = alloc_base(c, c->arena, &base);
+  if (st != NBODY_OK) return st;
+  CK(cudaIpcGetMemHandle(&d.ipc, const_cast<char*>(base)));
+  d.offset = uint64_t(c->arena - base);
   d.n = c->n;
   d.arena_bytes = c->arena_bytes;
   d.magic = kPeerMagic;
@@ -1269,7 +1478,7 @@ nbody_status nbody_attach_peers(nbody_ctx* c, const void* handles, int rank, int
       return fail(c, NBODY_ECUDA, "cudaIpcOpenMemHandle(peer " + std::to_string(q) + "): " + cudaGetErrorString(e));
     }
     c->peer_map[q] = p;
-    base[q] = static_cast<char*>(p);
+    base[q] = static_cast<char*>(p) + d.offset;
   }
   return attach_peer_bases(c, base, rank, world);
 }
@@ -1464,13 +1673,13 @@ void nbody_destroy(nbody_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   drop_graph(c);
 #ifdef NBODY_WITH_NCCL
-  if (c->comm) ncclCommDestroy(c->comm);
+  if (c->comm && !c->comm_borrowed) ncclCommDestroy(c->comm);
 #endif
   for (auto& p : c->peer_map)
     if (p) cudaIpcCloseMemHandle(p);
-  if (c->arena) cudaFree(c->arena);
-  if (c->quad_arena) cudaFree(c->quad_arena);
-  if (c->arena64) cudaFree(c->arena64);
+  dev_free(c, c->arena);
+  dev_free(c, c->quad_arena);
+  dev_free(c, c->arena64);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
   for (cudaStream_t cs : {c->cstream, c->ostream})
@@ -1481,7 +1690,7 @@ void nbody_destroy(nbody_ctx* c) {
   for (int k = 0; k < 2; ++k)
     for (cudaEvent_t e : {c->ev_in_copied[k], c->ev_in_used[k], c->ev_out_ready[k], c->ev_out_copied[k]})
       if (e) cudaEventDestroy(e);
-  if (c->xfer) cudaFree(c->xfer);
+  dev_free(c, c->xfer);
   if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
   if (c->own_stream) cudaStreamDestroy(c->own_stream);
   cudaGetLastError();

@@ -149,6 +149,12 @@ constexpr int kK6Stats = 37;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
+// NEXT-1 fp32 all-pairs (k_allpairs.cu); target slots of ids (k_direct.cu)
+void launch_target_slots(const float4* vi, int64_t n, const int64_t* ids, int64_t nt, uint32_t* slot_of,
+                         uint32_t* tslot, cudaStream_t s);
+int64_t allpairs_chunks(int64_t n, int64_t nt, int nsm);
+void launch_allpairs32(const float4* pm, int64_t n, const uint32_t* tslot, int64_t nt, float eps2, int64_t chunks,
+                       double4* part, double* out, cudaEvent_t ev0, cudaEvent_t ev1, cudaStream_t s);
 int64_t direct_chunks(int64_t n, int64_t nt);
 void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t* ids, int64_t nt, double eps2,
                    uint32_t* slot_of, uint32_t* tslot, double4* part, double* out, cudaStream_t s);

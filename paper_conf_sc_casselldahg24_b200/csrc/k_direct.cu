@@ -87,11 +87,17 @@ int64_t direct_chunks(int64_t n, int64_t nt) {
   return chunks;
 }
 
-void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t* ids, int64_t nt, double eps2,
-                   uint32_t* slot_of, uint32_t* tslot, double4* part, double* out, cudaStream_t s) {
+void launch_target_slots(const float4* vi, int64_t n, const int64_t* ids, int64_t nt, uint32_t* slot_of,
+                         uint32_t* tslot, cudaStream_t s) {
   if (nt <= 0) return;
   k_slot_of_id<<<unsigned((n + 255) / 256), 256, 0, s>>>(vi, n, slot_of);
   k_gather_u32<<<unsigned((nt + 255) / 256), 256, 0, s>>>(slot_of, ids, nt, tslot);
+}
+
+void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t* ids, int64_t nt, double eps2,
+                   uint32_t* slot_of, uint32_t* tslot, double4* part, double* out, cudaStream_t s) {
+  if (nt <= 0) return;
+  launch_target_slots(vi, n, ids, nt, slot_of, tslot, s);
   const int64_t chunks = direct_chunks(n, nt);
   const int64_t chunk = (n + chunks - 1) / chunks;
   dim3 grid(unsigned((nt + kDThreads - 1) / kDThreads), unsigned(chunks));

@@ -61,7 +61,11 @@ class NBody:
 
     def __init__(self, n: int, theta: float = 0.5, eps: float = 1e-3, dt: float = 1e-3, *, key_bits: int = 16,
                  stream=None, use_graph: bool = True, traversal: int = 0, device=None, multipole: int = 1,
-                 balance: bool = False, precision: int = 32):
+                 balance: bool = False, precision: int = 32, workspace=None):
+        """``workspace``: optional caller-owned device buffer (a CUDA uint8
+        torch tensor, at least ``NBody.workspace_bytes(n, ...)`` bytes) the
+        context carves all its device memory from (nbody_create_ws); the
+        caller keeps it alive while the context lives."""
         self.lib = _capi.load()
         self.n = int(n)
         if device is None:  # follow PyTorch's current device when torch has one
@@ -76,9 +80,15 @@ class NBody:
             if st != 0:
                 raise _capi.NBodyError(st, f"nbody_select_device({device}) failed")
         h = C.c_void_p()
-        st = self.lib.nbody_create(self.n, float(theta), float(eps), float(dt), C.byref(h))
+        if workspace is None:
+            st = self.lib.nbody_create(self.n, float(theta), float(eps), float(dt), C.byref(h))
+        else:
+            nbytes = workspace.numel() * workspace.element_size()
+            st = self.lib.nbody_create_ws(self.n, float(theta), float(eps), float(dt), _ptr(workspace), nbytes,
+                                          C.byref(h))
         if st != 0:
-            raise _capi.NBodyError(st, "nbody_create failed")
+            raise _capi.NBodyError(st, "nbody_create failed" if workspace is None else "nbody_create_ws failed")
+        self.workspace = workspace
         self.h = h
         self.set_option(_capi.NBODY_OPT_KEY_BITS, key_bits)
         self.set_option(_capi.NBODY_OPT_USE_GRAPH, int(use_graph))
@@ -92,6 +102,15 @@ class NBody:
             self.set_option(_capi.NBODY_OPT_PRECISION, self.precision)
         if stream is not None:
             self.set_option(_capi.NBODY_OPT_STREAM, int(stream))
+
+    @staticmethod
+    def workspace_bytes(n: int, world: int = 1, key_bits: int = 16, features: int = 0) -> int:
+        """Device bytes a context for n bodies needs (nbody_workspace_bytes_ex);
+        features: NBODY_WS_QUAD | NBODY_WS_XFER | NBODY_WS_FP64."""
+        b = _capi.load().nbody_workspace_bytes_ex(int(n), int(world), int(key_bits), int(features))
+        if b == 0:
+            raise ValueError("invalid arguments to nbody_workspace_bytes_ex")
+        return int(b)
 
     # -- lifecycle ---------------------------------------------------------
     def close(self):
@@ -219,6 +238,17 @@ class NBody:
         self._ck(self.lib.nbody_direct_accel(self.h, _ptr(ids), len(ids), _ptr(out)))
         return out
 
+    def allpairs_accel(self, ids, timed: bool = False):
+        """NEXT-1 fp32 all-pairs accelerations (fp64 output) of the given body
+        ids against all n sources; with timed=True also the kernel's device
+        time in ms."""
+        ids = np.ascontiguousarray(ids, np.int64)
+        out = np.empty((len(ids), 3), np.float64)
+        ms = C.c_float(0.0)
+        self._ck(self.lib.nbody_allpairs_accel(self.h, _ptr(ids), len(ids), _ptr(out),
+                                               C.byref(ms) if timed else None))
+        return (out, ms.value) if timed else out
+
     # -- multi-GPU ---------------------------------------------------------
     def set_partition(self, rank: int, world: int):
         self._ck(self.lib.nbody_set_partition(self.h, int(rank), int(world)))
@@ -241,6 +271,19 @@ class NBody:
         rank 0 creates the unique id, the process group broadcasts it."""
         from .dist import broadcast_unique_id
         self.attach_nccl(broadcast_unique_id(rank, group), rank, world)
+
+    def attach_comm(self, comm_ptr: int, rank: int, world: int):
+        """Run the exchange on an existing ncclComm_t (nbody_attach_comm)."""
+        self._ck(self.lib.nbody_attach_comm(self.h, C.c_void_p(int(comm_ptr)), int(rank), int(world)))
+
+    def attach_torch_comm(self, group=None):
+        """Use torch.distributed's own NCCL communicator of this device (the
+        process group must be NCCL and eagerly initialised with device_id)."""
+        import torch
+        import torch.distributed as dist
+        g = group if group is not None else dist.group.WORLD
+        backend = g._get_backend(torch.device("cuda", torch.cuda.current_device()))
+        self.attach_comm(backend._comm_ptr(), dist.get_rank(g), dist.get_world_size(g))
 
     # fused update + exchange over peer memory (nbody_attach_peers)
     def peer_handle(self) -> bytes:

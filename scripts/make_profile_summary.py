@@ -78,7 +78,10 @@ def main(tag):
             to_bytes(k["dram__bytes_write.sum"], u["dram__bytes_write.sum"])
         d = {"tag": tag, "kernel": k["kernel"], "command": "ncu --set full --clock-control none --import-source on "
              "-k regex:k_force -s 1 -c 1 python scripts/run_pass.py --passes 2 (disks N=1e7, theta=0.5)",
-             "dram_bytes_per_launch": traffic, "metrics": {m: k[m] for m in METRICS}, "units": u}
+             "dram_bytes_per_launch": traffic, "metrics": {m: k[m] for m in METRICS}, "units": u,
+             # the configuration of the capture (bench.py uses a capture's traffic only for the same one)
+             "config": {"workload": "disks", "n": 10_000_000, "theta": 0.5, "precision": 32, "multipole": 1,
+                        "key_bits": 16}}
         with open(os.path.join(PROF, f"{tag}_force_ncu.json"), "w") as f:
             json.dump(d, f, indent=1)
     br = os.path.join(OUT, f"build_{tag}.ncu-rep")

@@ -58,7 +58,10 @@ s.step(3)
 s.sync()
 print("tree reuse: ok", flush=True)
 s.close()
-ranks = [NBody(n, 0.5, 1e-3, 1e-3, use_graph=False, device=0, balance=True) for _ in range(2)]
+# the sanitizer serialises kernels, so ranks on one GPU whose device barriers
+# wait for each other would deadlock: one rank exercises the exchange kernels
+# (scatter stores, barriers, partition) against itself
+ranks = [NBody(n, 0.5, 1e-3, 1e-3, use_graph=False, device=0, balance=True) for _ in range(1)]
 NBody.attach_peers_local(ranks)
 for r in ranks:
     r.set_bodies(pos, vel, mass)
@@ -67,7 +70,7 @@ for _ in range(2):
         r.step(1)
 for r in ranks:
     r.sync()
-print("peer exchange x2 (balanced): ok", flush=True)
+print("peer exchange kernels, one rank (balanced): ok", flush=True)
 for r in ranks:
     r.close()
 ids = np.arange(0, n, 97)

@@ -78,3 +78,31 @@ def test_oracle_and_cuda_path_share_nothing():
             assert "from oracle" not in open(os.path.join(pkg, f)).read()
     otxt = open(os.path.join(ROOT, "oracle", "bvh_oracle.cpp")).read()
     assert "#include \"" not in otxt and "csrc" not in otxt.replace("paper_conf_sc_casselldahg24_b200/csrc", "")
+
+
+def test_workspace_bytes_host_side(lib):
+    """nbody_workspace_bytes is host-only (no device needed): one layout per N
+    (sizes fixed by N), every world and key width; 0 on bad
+    arguments; the optional buffers add their documented sizes."""
+    from paper_conf_sc_casselldahg24_b200 import _capi
+    f = lib.nbody_workspace_bytes
+    fx = lib.nbody_workspace_bytes_ex
+    for n in (1, 1000, 10_000_000):
+        base = f(n, 1, 16)
+        assert base > 0 and base % 256 == 0
+        assert f(n, 8, 0) == base and f(n, 256, 21) == base
+        L = max(0, (n - 1).bit_length())
+        inner = 1 << L
+        assert fx(n, 1, 16, _capi.NBODY_WS_QUAD) - base >= 80 * inner
+        assert fx(n, 1, 16, _capi.NBODY_WS_XFER) - base >= 80 * n
+        assert fx(n, 1, 16, _capi.NBODY_WS_FP64) - base >= 128 * n
+        assert fx(n, 1, 16, 7) == (fx(n, 1, 16, 1) + fx(n, 1, 16, 2) + fx(n, 1, 16, 4) - 2 * base)
+    # about 300 B of state + keys + sort per body and about 100 B per tree id at 10^7
+    assert 3e9 < f(10_000_000, 1, 16) < 6e9
+    assert f(2000, 1, 16) > f(1000, 1, 16)
+    for bad in ((0, 1, 16), (1 << 30, 1, 16), (10, 0, 16), (10, 257, 16), (10, 1, 22), (10, 1, -1)):
+        assert f(*bad) == 0
+    assert fx(10, 1, 16, 8) == 0
+    h = C.c_void_p()
+    assert lib.nbody_create_ws(10, 0.5, 1e-3, 1e-3, None, 1 << 20, C.byref(h)) == -1 and not h.value
+    assert lib.nbody_attach_comm(None, None, 0, 1) == -1
