@@ -695,6 +695,20 @@ nbody_status nbody_select_device(int device) {
   return cudaSetDevice(device) == cudaSuccess ? NBODY_OK : NBODY_ECUDA;
 }
 
+static void preload_all() {
+  static bool done = false;  // per process; kernels are loaded per context, and the library uses one device context
+  if (done) return;
+  done = true;
+  preload_allpairs();
+  preload_bbox_keys();
+  preload_build();
+  preload_direct();
+  preload_exchange();
+  preload_force();
+  preload_update();
+  preload_sort();
+}
+
 static nbody_status create_impl(int64_t n, double theta, double eps, double dt, void* ws, size_t ws_bytes,
                                 nbody_ctx** out) {
   if (!out) return NBODY_EINVAL;
@@ -732,6 +746,7 @@ static nbody_status create_impl(int64_t n, double theta, double eps, double dt, 
   for (auto& e : c->ev)
     if (cudaEventCreate(&e) != cudaSuccess) return bail(NBODY_ECUDA);
   c->stream = c->own_stream;
+  preload_all();
   nbody_status s = allocate(c);
   if (s != NBODY_OK) return bail(s);
   set_part(c, 0, 1);

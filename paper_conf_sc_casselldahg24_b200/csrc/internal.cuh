@@ -145,10 +145,28 @@ void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s);
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
-constexpr int kK6Stats = 37;
+constexpr int kK6Stats = 42;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
+// Lazy module loading (the CUDA 12 default) loads a kernel at its first
+// launch, and the loader can wait for the device to go idle; a context whose
+// device barrier spins on another context of the same process (the fused
+// peer exchange with graphs off) would then deadlock.  preload_*() touch
+// every kernel once (cudaFuncGetAttributes), called at nbody_create.
+template <class F>
+inline void touch(F* f) {
+  cudaFuncAttributes a;
+  if (cudaFuncGetAttributes(&a, f) != cudaSuccess) cudaGetLastError();
+}
+void preload_allpairs();
+void preload_bbox_keys();
+void preload_build();
+void preload_direct();
+void preload_exchange();
+void preload_force();
+void preload_update();
+void preload_sort();
 // NEXT-1 fp32 all-pairs (k_allpairs.cu); target slots of ids (k_direct.cu)
 void launch_target_slots(const float4* vi, int64_t n, const int64_t* ids, int64_t nt, uint32_t* slot_of,
                          uint32_t* tslot, cudaStream_t s);

@@ -166,4 +166,12 @@ void launch_allpairs32(const float4* pm, int64_t n, const uint32_t* tslot, int64
   k_allpairs_reduce<<<unsigned((nt + 255) / 256), 256, 0, s>>>(part, nt, int64_t(grid.y), out);
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_allpairs() {
+  touch(k_allpairs32<false>);
+  touch(k_allpairs32<true>);
+  touch(k_allpairs_reduce);
+}
+
 }  // namespace nb

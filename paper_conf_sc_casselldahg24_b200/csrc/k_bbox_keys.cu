@@ -369,4 +369,18 @@ void launch_keys_f64(const double4* pm, int64_t n, const GridInfo* g, void* keys
         <<<keys_grid(n), kKeysThreads, 0, s>>>(pm, n, g, static_cast<unsigned long long*>(keys), ghist, passes);
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_bbox_keys() {
+  touch(k_bbox_final);
+  touch(k_bbox_final_f64);
+  touch(k_bbox_partial);
+  touch(k_bbox_partial_f64);
+  touch(k_keys<uint32_t, float4>);
+  touch(k_keys<uint32_t, double4>);
+  touch(k_keys<unsigned long long, float4, 16, 6>);
+  touch(k_keys<unsigned long long, float4>);
+  touch(k_keys<unsigned long long, double4>);
+}
+
 }  // namespace nb

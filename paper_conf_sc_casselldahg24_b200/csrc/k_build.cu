@@ -395,4 +395,18 @@ void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s) {
     k_build_level<<<unsigned((t.count[l] + 255) / 256), 256, 0, s>>>(t, l);
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_build() {
+  touch(k_build_upper<false>);
+  touch(k_build_upper<true>);
+  touch(k_build_fused<false, false>);
+  touch(k_build_fused<false, true>);
+  touch(k_build_fused<true, false>);
+  touch(k_build_level);
+  touch(k_build_level1);
+  touch(k_permute);
+  touch(k_permute_f64);
+}
+
 }  // namespace nb

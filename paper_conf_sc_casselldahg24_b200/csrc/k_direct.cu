@@ -105,4 +105,13 @@ void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t*
   k_direct_reduce<<<unsigned((nt + 255) / 256), 256, 0, s>>>(part, nt, chunks, out);
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_direct() {
+  touch(k_direct_partial);
+  touch(k_direct_reduce);
+  touch(k_gather_u32);
+  touch(k_slot_of_id);
+}
+
 }  // namespace nb

@@ -567,6 +567,7 @@ __device__ __forceinline__ float warp_maxf(float v) {
 }
 
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
+__device__ __forceinline__ float inf_stat() { return __int_as_float(0x7f800000); }
 
 // Transposed-phase filter of the fp64 opening test.
 // With g the group reference point (fp32), c~ = com64 - g, x~ = x - g (exact
@@ -840,6 +841,20 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
 #ifdef NBODY_K6_STATS
   unsigned long long st[kK6Stats] = {};
   int sq[4] = {0, 0, 0, 0}, sh[2] = {0, 0}, s8[8] = {}, s16[16] = {}, s32 = 0;
+  int lq[4] = {0, 0, 0, 0}, lh[2] = {0, 0}, lg = 0;  // quarter-local / half-local / general partial entries
+  // boxes of the 128- and 256-target super-groups (block-level box phase study)
+  float sb[2][6];
+  for (int w2 = 0; w2 < 2; ++w2) {
+    const int64_t span = w2 ? 256 : 128;
+    const int64_t g0 = tb + ((k0 - tb) / span) * span;
+    float lo[3] = {inf_stat(), inf_stat(), inf_stat()}, hi[3] = {-inf_stat(), -inf_stat(), -inf_stat()};
+    for (int64_t kk = g0 + lane; kk < g0 + span && kk < te; kk += 32) {
+      const float4 q = P.leaves[kk];
+      lo[0] = fminf(lo[0], q.x); lo[1] = fminf(lo[1], q.y); lo[2] = fminf(lo[2], q.z);
+      hi[0] = fmaxf(hi[0], q.x); hi[1] = fmaxf(hi[1], q.y); hi[2] = fmaxf(hi[2], q.z);
+    }
+    for (int d = 0; d < 3; ++d) { sb[w2][d] = warp_minf(lo[d]); sb[w2][3 + d] = warp_maxf(hi[d]); }
+  }
 #endif
   K6STAT(0, 1);
   if (lane == 0) S.astk[0] = 1u;
@@ -904,6 +919,16 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       for (int j = 0; j < 8; ++j) s8[j] += __popc(__ballot_sync(kFull, part && ((msk >> (4 * j)) & 0xfu)));
       for (int j = 0; j < 16; ++j) s16[j] += __popc(__ballot_sync(kFull, part && ((msk >> (2 * j)) & 0x3u)));
       s32 += part ? 0 : 0;
+      {
+        const bool ql = part && (((msk & 0xffu) == msk) || ((msk & 0xff00u) == msk) || ((msk & 0xff0000u) == msk) ||
+                                 ((msk & 0xff000000u) == msk));
+        const bool hl = part && !ql && (((msk & 0xffffu) == msk) || ((msk >> 16) << 16) == msk);
+        const int q = msk & 0xffffu ? (msk & 0xffu ? 0 : 1) : (msk & 0xff0000u ? 2 : 3);
+        for (int j = 0; j < 4; ++j) lq[j] += __popc(__ballot_sync(kFull, ql && q == j));
+        lh[0] += __popc(__ballot_sync(kFull, hl && (msk & 0xffffu)));
+        lh[1] += __popc(__ballot_sync(kFull, hl && !(msk & 0xffffu)));
+        lg += __popc(__ballot_sync(kFull, part && !ql && !hl));
+      }
       for (int j = 0; j < 32; ++j) {
         const uint32_t mj = __shfl_sync(kFull, msk, j);
         const bool pj = __shfl_sync(kFull, part, j);
@@ -931,6 +956,10 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       K6STAT(12, 1);
       K6STAT(13, (np + 1) >> 1);
 #ifdef NBODY_K6_STATS
+      K6STAT(37, max(max(lq[0], lq[1]), max(lq[2], lq[3])));
+      K6STAT(38, max(lh[0], lh[1]));
+      K6STAT(39, lg);
+      lq[0] = lq[1] = lq[2] = lq[3] = lh[0] = lh[1] = lg = 0;
       K6STAT(22, max(max(sq[0], sq[1]), max(sq[2], sq[3])));
       K6STAT(23, max(sh[0], sh[1]));
       sq[0] = sq[1] = sq[2] = sq[3] = sh[0] = sh[1] = 0;
@@ -1116,6 +1145,16 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
             cls = 3;
             K6STAT(36, dmax2 * (1.f + 4e-6f) < c.x);  // an all-open node handed to T by the capacity guard
           }
+#ifdef NBODY_K6_STATS
+          for (int w2 = 0; w2 < 2; ++w2) {  // would the 128 / 256-target super-group box decide this node?
+            const float bx0 = sb[w2][0] - r.x, bx1 = r.x - sb[w2][3], by0 = sb[w2][1] - r.y, by1 = r.y - sb[w2][4];
+            const float bz0 = sb[w2][2] - r.z, bz1 = r.z - sb[w2][5];
+            const float mx = fmaxf(0.f, fmaxf(bx0, bx1)), my = fmaxf(0.f, fmaxf(by0, by1)), mz = fmaxf(0.f, fmaxf(bz0, bz1));
+            const float Mx = fmaxf(fabsf(bx0), fabsf(bx1)), My = fmaxf(fabsf(by0), fabsf(by1)), Mz = fmaxf(fabsf(bz0), fabsf(bz1));
+            const float bmin2 = fmaf(mz, mz, fmaf(my, my, mx * mx)), bmax2 = fmaf(Mz, Mz, fmaf(My, My, Mx * Mx));
+            K6STAT(40 + w2, bmin2 * (1.f - 4e-6f) > c.y || bmax2 * (1.f + 4e-6f) < c.x);
+          }
+#endif
         }
       }
       uint32_t msk = amask;
@@ -1177,6 +1216,20 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
     else
       k_force_grouped<false, true, false><<<grid, 32 * kV0Warps, 0, s>>>(p);
   }
+}
+
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_force() {
+  touch(k_force_grouped<false, false, false>);
+  touch(k_force_grouped<false, false, true>);
+  touch(k_force_grouped<false, true, false>);
+  touch(k_force_grouped<true, false, false>);
+  touch(k_force_grouped<true, false, true>);
+  touch(k_force_grouped<true, true, false>);
+  touch(k_force_maskstack<false>);
+  touch(k_force_maskstack<true>);
+  touch(k_force_skiplist);
 }
 
 }  // namespace nb

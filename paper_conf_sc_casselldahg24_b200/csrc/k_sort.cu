@@ -314,4 +314,19 @@ int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaSt
   return p.passes & 1;
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_sort() {
+  touch(k_hist<uint32_t>);
+  touch(k_hist<unsigned long long>);
+  touch(k_onesweep<uint32_t, false, false>);
+  touch(k_onesweep<uint32_t, false, true>);
+  touch(k_onesweep<uint32_t, true, false>);
+  touch(k_onesweep<uint32_t, true, true>);
+  touch(k_onesweep<unsigned long long, false, false>);
+  touch(k_onesweep<unsigned long long, false, true>);
+  touch(k_onesweep<unsigned long long, true, false>);
+  touch(k_onesweep<unsigned long long, true, true>);
+}
+
 }  // namespace nb

@@ -178,4 +178,19 @@ void launch_scatter_by_id1_f64(const uint32_t* src, const double4* vi, int64_t n
   k_scatter1_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
 }
 
+
+// Load every kernel of this file now (see preload_all in capi.cu).
+void preload_update() {
+  touch(k_fill2);
+  touch(k_leapfrog);
+  touch(k_leapfrog_f64);
+  touch(k_pack);
+  touch(k_pack_f64);
+  touch(k_scatter1);
+  touch(k_scatter1_f64);
+  touch(k_scatter3);
+  touch(k_scatter3_f64<double>);
+  touch(k_scatter3_f64<float>);
+}
+
 }  // namespace nb

@@ -242,7 +242,13 @@ class NBody:
         """NEXT-1 fp32 all-pairs accelerations (fp64 output) of the given body
         ids against all n sources; with timed=True also the kernel's device
         time in ms."""
-        ids = np.ascontiguousarray(ids, np.int64)
+        if hasattr(ids, "data_ptr"):  # a torch tensor (host or device): int64, contiguous
+            import torch
+            if ids.dtype != torch.int64:
+                raise ValueError("ids must be int64")
+            ids = ids.contiguous()
+        else:
+            ids = np.ascontiguousarray(ids, np.int64)
         out = np.empty((len(ids), 3), np.float64)
         ms = C.c_float(0.0)
         self._ck(self.lib.nbody_allpairs_accel(self.h, _ptr(ids), len(ids), _ptr(out),
