@@ -289,6 +289,10 @@ size_t f64_bytes_for(int64_t n, int nsm) {
 
 // Device memory for the context: from the caller's workspace (create_ws),
 // else cudaMalloc.  `what` names the buffer in the error.
+// The memory is zeroed once: some kernels load whole sibling pairs or
+// vectors that include never-written slots (the missing right sibling at the
+// ragged end of a level) and discard them; zero-filled, those reads are of
+// defined memory (compute-sanitizer initcheck is clean).
 nbody_status dev_alloc(nbody_ctx* c, size_t bytes, void** out, const char* what) {
   *out = nullptr;
   bytes = align_up(bytes);
@@ -299,14 +303,16 @@ nbody_status dev_alloc(nbody_ctx* c, size_t bytes, void** out, const char* what)
                                        "with the optional buffers)");
     *out = c->ws + c->ws_used;
     c->ws_used += bytes;
-    return NBODY_OK;
+  } else {
+    const cudaError_t e = cudaMalloc(out, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      *out = nullptr;
+      return fail(c, NBODY_ENOMEM, std::string(what) + ": cudaMalloc of " + std::to_string(bytes) + " bytes failed");
+    }
   }
-  const cudaError_t e = cudaMalloc(out, bytes);
-  if (e != cudaSuccess) {
-    cudaGetLastError();
-    *out = nullptr;
-    return fail(c, NBODY_ENOMEM, std::string(what) + ": cudaMalloc of " + std::to_string(bytes) + " bytes failed");
-  }
+  CK(cudaMemsetAsync(*out, 0, bytes, c->stream ? c->stream : cudaStreamLegacy));
+  CK(cudaStreamSynchronize(c->stream ? c->stream : cudaStreamLegacy));
   return NBODY_OK;
 }
 void dev_free(nbody_ctx* c, void* p) {

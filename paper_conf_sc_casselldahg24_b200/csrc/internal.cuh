@@ -145,7 +145,7 @@ void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s);
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
-constexpr int kK6Stats = 42;
+constexpr int kK6Stats = 46;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------

@@ -1111,6 +1111,10 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       na = base;
       const bool guard = na + 64 > kCapA;
       int cls = 0;  // 1 dense, 2 expand, 3 transposed
+#ifdef NBODY_K6_STATS
+      bool guard_open = false;
+      int sdec[2] = {0, 0};
+#endif
       float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
       bool two = false;
       if (has) {
@@ -1143,7 +1147,9 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
             two = ((2u * g + 1u) << (l - 1)) - leaf0 < n;
           } else {
             cls = 3;
-            K6STAT(36, dmax2 * (1.f + 4e-6f) < c.x);  // an all-open node handed to T by the capacity guard
+#ifdef NBODY_K6_STATS
+            guard_open = dmax2 * (1.f + 4e-6f) < c.x;  // an all-open node handed to T by the capacity guard
+#endif
           }
 #ifdef NBODY_K6_STATS
           for (int w2 = 0; w2 < 2; ++w2) {  // would the 128 / 256-target super-group box decide this node?
@@ -1152,11 +1158,20 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
             const float mx = fmaxf(0.f, fmaxf(bx0, bx1)), my = fmaxf(0.f, fmaxf(by0, by1)), mz = fmaxf(0.f, fmaxf(bz0, bz1));
             const float Mx = fmaxf(fabsf(bx0), fabsf(bx1)), My = fmaxf(fabsf(by0), fabsf(by1)), Mz = fmaxf(fabsf(bz0), fabsf(bz1));
             const float bmin2 = fmaf(mz, mz, fmaf(my, my, mx * mx)), bmax2 = fmaf(Mz, Mz, fmaf(My, My, Mx * Mx));
-            K6STAT(40 + w2, bmin2 * (1.f - 4e-6f) > c.y || bmax2 * (1.f + 4e-6f) < c.x);
+            sdec[w2] = bmin2 * (1.f - 4e-6f) > c.y ? 1 : bmax2 * (1.f + 4e-6f) < c.x ? 2 : 0;
           }
 #endif
         }
       }
+#ifdef NBODY_K6_STATS
+      K6STAT(36, __reduce_add_sync(kFull, guard_open ? 1u : 0u));
+      K6STAT(40, __reduce_add_sync(kFull, sdec[0] != 0 ? 1u : 0u));
+      K6STAT(41, __reduce_add_sync(kFull, sdec[1] != 0 ? 1u : 0u));
+      K6STAT(42, __reduce_add_sync(kFull, sdec[0] == 1 ? 1u : 0u));
+      K6STAT(43, __reduce_add_sync(kFull, has && g < leaf0 ? 1u : 0u));
+      K6STAT(44, __reduce_add_sync(kFull, cls == 1 && g < leaf0 ? 1u : 0u));
+      K6STAT(45, __reduce_add_sync(kFull, cls == 2 ? 1u : 0u));
+#endif
       uint32_t msk = amask;
       if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
       append(cls == 1, r, msk, g < leaf0 ? g : 0u, g);
