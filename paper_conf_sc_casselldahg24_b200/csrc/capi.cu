@@ -112,6 +112,10 @@ struct nbody_ctx {
   uint32_t* gcost = nullptr;        // [ceil(n/32)] interactions per 32-slot group, last pass
   int64_t* dpart = nullptr;         // [kMaxPeers + 1] slot boundaries of the next pass
   int64_t* dpart_used = nullptr;    // [kMaxPeers + 1] boundaries of the last pass
+  // K6a super-group lists (k_force.cu)
+  uint32_t* sg_acc = nullptr;
+  uint32_t* sg_fr = nullptr;
+  int2* sg_cnt = nullptr;
   // pipelined host transfers (nbody_set_bodies_async / nbody_get_positions_async)
   cudaStream_t cstream = nullptr;   // copy stream, host -> device
   cudaStream_t ostream = nullptr;   // copy stream, device -> host (separate: it waits for steps)
@@ -246,6 +250,9 @@ int arena_plan(int64_t n, int nsm, size_t* sz) {
   sz[k++] = 16 * size_t(inner);                     // tf
   sz[k++] = 4 * size_t(n / 32 + 1);                 // gcost
   sz[k++] = 512;                                    // exchange flags, epochs, error, partitions
+  sz[k++] = 4 * size_t(kSGAcc) * size_t(sg_groups(n));  // K6a super-group lists: accepted
+  sz[k++] = 4 * size_t(kSGFr) * size_t(sg_groups(n));   //   frontier
+  sz[k++] = 8 * size_t(sg_groups(n)) + 8;               //   counts
   return k;
 }
 
@@ -365,6 +372,9 @@ nbody_status allocate(nbody_ctx* c) {
   c->xflags = (unsigned*)take();
   c->xepoch = c->xflags + kBarrierSlots * kMaxPeers;
   c->xerr = reinterpret_cast<int*>(c->xepoch + kBarrierSlots);
+  c->sg_acc = (uint32_t*)take();
+  c->sg_fr = (uint32_t*)take();
+  c->sg_cnt = (int2*)take();
   c->dpart = reinterpret_cast<int64_t*>(reinterpret_cast<char*>(c->xflags) + 128);
   c->dpart_used = c->dpart + kMaxPeers + 1;
   c->arena_bytes = total;
@@ -535,6 +545,14 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     fp.cap = std::min(n, 32 * cap_groups);
     fp.xp = c->peers;
   }
+  int sg_kernels = 0;
+  if (c->traversal == 0 && kSG > 0) {  // K6a, then K6 continues from its lists
+    fp.sg_acc = c->sg_acc;
+    fp.sg_fr = c->sg_fr;
+    fp.sg_cnt = c->sg_cnt;
+    launch_force_sgroups(fp, s);
+    sg_kernels = 1;
+  }
   launch_force(fp, c->traversal, s);
   CK(mark(4));
   if (integrate && c->xpeer) {
@@ -584,7 +602,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   CK(mark(5));
   c->ev_valid = tm;
   // K1 2 + K2 (with the digit histograms) 1 + K3 passes + K4 1 + K5 + K6 1 + K7 1
-  c->kernels_per_step = front_kernels + build_kernels + 1 + (integrate ? 1 : 0) + x_kernels;
+  c->kernels_per_step = front_kernels + build_kernels + 1 + sg_kernels + (integrate ? 1 : 0) + x_kernels;
   CK(cudaGetLastError());
   return NBODY_OK;
 }

@@ -96,7 +96,27 @@ struct ForceParams {
   int part_rank = 0;
   int64_t cap = 0;
   PeerTable xp{};
+  // Super-group pre-pass (k_force.cu K6a): per super-group of kSG
+  // consecutive owned targets, the nodes every one of them accepts (acc) and
+  // the frontier of nodes its box does not decide (fr); cnt = (n_acc, n_fr),
+  // (-1, -1) after an overflow (the warps then start from the root).
+  uint32_t* sg_acc = nullptr;
+  uint32_t* sg_fr = nullptr;
+  int2* sg_cnt = nullptr;
 };
+
+// Super-group size and list capacities of K6a (k_force.cu).
+#ifndef NBODY_SG
+#define NBODY_SG 256
+#endif
+#ifndef NBODY_SG_ACC
+#define NBODY_SG_ACC 2048
+#endif
+#ifndef NBODY_SG_FR
+#define NBODY_SG_FR 1024
+#endif
+constexpr int kSG = NBODY_SG, kSGAcc = NBODY_SG_ACC, kSGFr = NBODY_SG_FR;
+inline int64_t sg_groups(int64_t n) { return kSG > 0 ? (n + kSG - 1) / kSG + 1 : 0; }
 
 // ---- K1 / K2 --------------------------------------------------------------
 void launch_bbox_partial(const float4* pm, int64_t n, float* partial, int nblocks, cudaStream_t s);
@@ -144,6 +164,8 @@ void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s);
 
 // ---- K6 --------------------------------------------------------------------
 void launch_force(const ForceParams& p, int variant, cudaStream_t s);
+// K6a: the super-group lists of p (p.sg_* must be set); variant-0 K6 reads them.
+void launch_force_sgroups(const ForceParams& p, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
 constexpr int kK6Stats = 46;
 int force_stats(unsigned long long* out, int n);

@@ -550,6 +550,7 @@ struct alignas(16) V0Smem {
   uint32_t pmsk[kCapP];     // ... for the lanes in the mask
   uint32_t astk[kCapA];
   uint2 tstk[kT];     // (id, mask of the targets that reached it)
+  int sg_next, sg_nfr;  // super-group frontier: next entry, length (K6a)
   using QP = typename std::conditional<kQuad, QuadPair, char>::type;
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
   QP pq[kQuad ? kCapP / 2 : 1];
@@ -857,7 +858,24 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   }
 #endif
   K6STAT(0, 1);
-  if (lane == 0) S.astk[0] = 1u;
+  // Super-group lists (K6a): start from the frontier of this warp's super-
+  // group instead of the root, after the nodes every target of the super-
+  // group accepts (every target of this warp then accepts them too, and
+  // every frontier node was opened by all of them with all its ancestors,
+  // so the lists are the ones the walk from the root produces).
+  const uint32_t sgi = kSG > 0 ? uint32_t((k0 - tb) / kSG) : 0u;
+  int n_acc = -1;
+  {
+    int2 sgc = make_int2(-1, -1);
+    if (kSG > 0 && P.sg_cnt) sgc = P.sg_cnt[sgi];
+    n_acc = sgc.x;
+    if (lane == 0) {
+      if (sgc.x < 0) S.astk[0] = 1u;
+      S.sg_next = 0;
+      S.sg_nfr = sgc.x < 0 ? 0 : sgc.y;
+    }
+    if (sgc.x >= 0) na = 0;
+  }
   __syncwarp();
 
   // Append (record r, lane mask msk) to the dense lists: full when every
@@ -978,7 +996,26 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     __syncwarp();
   };
 
+  if (n_acc > 0) {  // the super-group's accepted nodes: full dense entries
+    const uint32_t* al = P.sg_acc + size_t(sgi) * kSGAcc;
+    for (int i = 0; i < n_acc; i += 32) {
+      const bool v = i + lane < n_acc;
+      const uint32_t g = v ? __ldg(al + i + lane) : 0u;
+      const float4 r = v ? __ldg(W.rec + g) : make_float4(0.f, 0.f, 0.f, 0.f);
+      append(v, r, amask, g, g);
+      flush(false);
+    }
+  }
   while (true) {
+    if (na == 0 && S.sg_next < S.sg_nfr) {  // refill the box stack from the super-group frontier
+      const int next = S.sg_next;
+      const int take = min(S.sg_nfr - next, kCapA - 64);
+      const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
+      for (int i = lane; i < take; i += 32) S.astk[i] = __ldg(fl + i);
+      __syncwarp();
+      if (lane == 0) S.sg_next = next + take;
+      na = take;
+    }
     if (nt >= 32 || (na == 0 && nt > 0)) {
       // ---- T: transposed classification of up to 32 (node, mask) entries
       const int take = nt < 32 ? nt : 32;
@@ -1199,7 +1236,130 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
 #endif
 }
 
+// ------------------------------------------------ super-group pre-pass ----
+// K6a: one warp per super-group of kSG consecutive owned targets classifies
+// nodes from the root against the super-group's bounding box with the box
+// phase's bounds (every target accepts / every target opens / neither):
+// accepted nodes go to acc, nodes it cannot decide (and leaves, whose
+// self-exclusion the force warps apply) to the frontier fr, nodes every
+// target opens are expanded.  Any warp of the super-group would decide
+// those nodes the same way with its own (smaller) box, so the force warps
+// take acc as full dense entries and continue from fr: the box-phase work
+// near the root is done once per kSG targets instead of once per 32.
+constexpr int kSGWarps = 4;
+
+template <bool kF64>
+__global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForceParams P) {
+  __shared__ uint32_t s_stk[kSGWarps][kCapA];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int64_t tb, te;
+  owned_range(P, tb, te);
+  const int64_t sgi = int64_t(blockIdx.x) * kSGWarps + w;
+  const int64_t g0 = tb + sgi * kSG;
+  if (g0 >= te) return;
+  const int64_t g1 = g0 + kSG < te ? g0 + kSG : te;
+  const float inf = __int_as_float(0x7f800000);
+  float lx = inf, ly = inf, lz = inf, hx = -inf, hy = -inf, hz = -inf;
+  for (int64_t k = g0 + lane; k < g1; k += 32) {
+    float x, y, z;
+    if constexpr (kF64) {  // the force kernel's fp32 rounding of the fp64 targets
+      const double4 q = P.leaves64[k];
+      x = float(q.x), y = float(q.y), z = float(q.z);
+    } else {
+      const float4 q = P.leaves[k];
+      x = q.x, y = q.y, z = q.z;
+    }
+    lx = fminf(lx, x), ly = fminf(ly, y), lz = fminf(lz, z);
+    hx = fmaxf(hx, x), hy = fmaxf(hy, y), hz = fmaxf(hz, z);
+  }
+  const float blx = warp_minf(lx), bly = warp_minf(ly), blz = warp_minf(lz);
+  const float bhx = warp_maxf(hx), bhy = warp_maxf(hy), bhz = warp_maxf(hz);
+  const float4* rec = in_reg(P.t.rec);
+  const float2* rc = in_reg(P.t.rc);
+  const uint32_t leaf0 = 1u << P.t.L, n = uint32_t(P.t.n);
+  const int L = P.t.L;
+  uint32_t* stk = s_stk[w];
+  uint32_t* acc = P.sg_acc + sgi * kSGAcc;
+  uint32_t* fr = P.sg_fr + sgi * kSGFr;
+  const uint32_t lt = (1u << lane) - 1u;
+  int na = 1, nacc = 0, nfr = 0;
+  if (lane == 0) stk[0] = 1u;
+  __syncwarp();
+  while (na > 0) {
+    const int take = na < 32 ? na : 32;
+    const int base = na - take;
+    const bool has = lane < take;
+    const uint32_t g = has ? stk[base + lane] : 0u;
+    __syncwarp();
+    na = base;
+    const bool guard = na + 64 > kCapA;
+    int cls = 0;  // 1 accepted by every target, 2 opened by every target, 3 frontier
+    bool two = false;
+    if (has) {
+      if (g >= leaf0) {
+        cls = 3;
+      } else {
+        // the force kernel's box-phase bounds
+        const float4 r = __ldg(rec + g);
+        const float2 c = __ldg(rc + g);
+        const float ax0 = blx - r.x, ax1 = r.x - bhx;
+        const float ay0 = bly - r.y, ay1 = r.y - bhy;
+        const float az0 = blz - r.z, az1 = r.z - bhz;
+        const float nx = fmaxf(0.f, fmaxf(ax0, ax1)), ny = fmaxf(0.f, fmaxf(ay0, ay1)),
+                    nz = fmaxf(0.f, fmaxf(az0, az1));
+        const float fx = fmaxf(fabsf(ax0), fabsf(ax1)), fy = fmaxf(fabsf(ay0), fabsf(ay1)),
+                    fz = fmaxf(fabsf(az0), fabsf(az1));
+        const float dmin2 = fmaf(nz, nz, fmaf(ny, ny, nx * nx));
+        const float dmax2 = fmaf(fz, fz, fmaf(fy, fy, fx * fx));
+        if (dmin2 * (1.f - 4e-6f) > c.y) {
+          cls = 1;
+        } else if (dmax2 * (1.f + 4e-6f) < c.x && !guard) {
+          cls = 2;
+          const int l = L - 31 + __clz(int(g));
+          two = ((2u * g + 1u) << (l - 1)) - leaf0 < n;
+        } else {
+          cls = 3;
+        }
+      }
+    }
+    const uint32_t ba = __ballot_sync(kFull, cls == 1), bf = __ballot_sync(kFull, cls == 3);
+    if (cls == 1) {
+      const int pos = nacc + __popc(ba & lt);
+      if (pos < kSGAcc) acc[pos] = g;
+    }
+    if (cls == 3) {
+      const int pos = nfr + __popc(bf & lt);
+      if (pos < kSGFr) fr[pos] = g;
+    }
+    nacc += __popc(ba);
+    nfr += __popc(bf);
+    if (nacc > kSGAcc || nfr > kSGFr) break;  // overflow: the force warps start from the root
+    const uint32_t b1 = __ballot_sync(kFull, cls == 2), b2 = __ballot_sync(kFull, cls == 2 && two);
+    if (cls == 2) {
+      const int pos = na + __popc(b1 & lt) + __popc(b2 & lt);
+      stk[pos] = 2u * g;
+      if (two) stk[pos + 1] = 2u * g + 1u;
+    }
+    na += __popc(b1) + __popc(b2);
+    __syncwarp();
+  }
+  if (lane == 0)
+    P.sg_cnt[sgi] = (nacc > kSGAcc || nfr > kSGFr) ? make_int2(-1, -1) : make_int2(nacc, nfr);
+}
+
 }  // namespace
+
+void launch_force_sgroups(const ForceParams& p, cudaStream_t s) {
+  if (kSG <= 0 || !p.sg_cnt) return;
+  const int64_t nt = p.part ? p.cap : p.t_end - p.t_begin;
+  if (nt <= 0) return;
+  const int64_t groups = (nt + kSG - 1) / kSG;
+  const unsigned grid = unsigned((groups + kSGWarps - 1) / kSGWarps);
+  if (p.t.rec64)
+    k_force_sgroups<true><<<grid, 32 * kSGWarps, 0, s>>>(p);
+  else
+    k_force_sgroups<false><<<grid, 32 * kSGWarps, 0, s>>>(p);
+}
 
 void launch_force(const ForceParams& p, int variant, cudaStream_t s) {
   const int64_t nt = p.part ? p.cap : p.t_end - p.t_begin;
@@ -1245,6 +1405,8 @@ void preload_force() {
   touch(k_force_maskstack<false>);
   touch(k_force_maskstack<true>);
   touch(k_force_skiplist);
+  touch(k_force_sgroups<false>);
+  touch(k_force_sgroups<true>);
 }
 
 }  // namespace nb
