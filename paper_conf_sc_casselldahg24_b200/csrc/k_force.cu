@@ -465,6 +465,9 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_V0_MINB
 #define NBODY_V0_MINB 8
 #endif
+#ifndef NBODY_SMEM_TOP
+#define NBODY_SMEM_TOP 0
+#endif
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 128
 #endif
@@ -785,6 +788,21 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   __shared__ V0Smem<kQuad, kF64> s_all[kV0Warps];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   V0Smem<kQuad, kF64>& S = s_all[w];
+#if NBODY_SMEM_TOP > 0
+  // design experiment (north star item 4, rejected: DESIGN.md "top levels in
+  // shared memory"): the records and filter thresholds of the top
+  // NBODY_SMEM_TOP levels (ids < 2^k) staged in shared memory for the box
+  // phase, loaded once per block
+  constexpr uint32_t kTop = 1u << NBODY_SMEM_TOP;
+  __shared__ float4 s_trec[kTop];
+  __shared__ float2 s_trc[kTop];
+  for (uint32_t i = threadIdx.x; i < kTop; i += blockDim.x)
+    if (i < (2u << P.t.L)) {
+      s_trec[i] = __ldg(P.t.rec + i);
+      s_trc[i] = __ldg(P.t.rc + i);
+    }
+  __syncthreads();
+#endif
   const float4* qf = kQuad ? in_reg(P.t.qf) : nullptr;
 #ifndef NBODY_GROUP
 #define NBODY_GROUP 32
@@ -863,7 +881,9 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // group accepts (every target of this warp then accepts them too, and
   // every frontier node was opened by all of them with all its ancestors,
   // so the lists are the ones the walk from the root produces).
-  const uint32_t sgi = kSG > 0 ? uint32_t((k0 - tb) / kSG) : 0u;
+  // super-groups are aligned to absolute slots (the same lists on any
+  // partition into ranks, hence results bit-identical to one GPU)
+  const uint32_t sgi = kSG > 0 ? uint32_t(k0 / kSG - tb / kSG) : 0u;
   int n_acc = -1;
   {
     int2 sgc = make_int2(-1, -1);
@@ -1165,8 +1185,14 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
           // |c32 - x|^2 within 5u each, so Dmin2 (1 - 4e-6) > hi => every
           // target's d2 > hi => all accept; Dmax2 (1 + 4e-6) < lo => all open
           // (DESIGN.md "fp32 filter").
+#if NBODY_SMEM_TOP > 0
+          const bool top = g < kTop;
+          r = top ? s_trec[g] : __ldg(W.rec + g);
+          const float2 c = top ? s_trc[g] : __ldg(W.rc + g);
+#else
           r = __ldg(W.rec + g);
           const float2 c = __ldg(W.rc + g);
+#endif
           const float ax0 = blx - r.x, ax1 = r.x - bhx;
           const float ay0 = bly - r.y, ay1 = r.y - bhy;
           const float az0 = blz - r.z, az1 = r.z - bhz;
@@ -1254,10 +1280,13 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   int64_t tb, te;
   owned_range(P, tb, te);
+  // list j of this rank: the super-group of absolute slots [g0, g0 + kSG),
+  // g0 = (tb / kSG + j) kSG, boxed over all its bodies (every rank holds the
+  // whole state) so that any partition sees the same lists as one GPU
   const int64_t sgi = int64_t(blockIdx.x) * kSGWarps + w;
-  const int64_t g0 = tb + sgi * kSG;
+  const int64_t g0 = (tb / kSG + sgi) * kSG;
   if (g0 >= te) return;
-  const int64_t g1 = g0 + kSG < te ? g0 + kSG : te;
+  const int64_t g1 = g0 + kSG < int64_t(P.t.n) ? g0 + kSG : int64_t(P.t.n);
   const float inf = __int_as_float(0x7f800000);
   float lx = inf, ly = inf, lz = inf, hx = -inf, hy = -inf, hz = -inf;
   for (int64_t k = g0 + lane; k < g1; k += 32) {
@@ -1353,7 +1382,7 @@ void launch_force_sgroups(const ForceParams& p, cudaStream_t s) {
   if (kSG <= 0 || !p.sg_cnt) return;
   const int64_t nt = p.part ? p.cap : p.t_end - p.t_begin;
   if (nt <= 0) return;
-  const int64_t groups = (nt + kSG - 1) / kSG;
+  const int64_t groups = (nt + kSG - 1) / kSG + 1;  // a range may straddle one more super-group
   const unsigned grid = unsigned((groups + kSGWarps - 1) / kSGWarps);
   if (p.t.rec64)
     k_force_sgroups<true><<<grid, 32 * kSGWarps, 0, s>>>(p);

@@ -8,8 +8,6 @@ import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
-from paper_conf_sc_casselldahg24_b200 import NBody  # noqa: E402
-from workloads import CONFIGS, generate  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="disks")
@@ -21,7 +19,21 @@ ap.add_argument("--traversal", type=int, default=0)
 ap.add_argument("--key-bits", type=int, default=16)
 ap.add_argument("--multipole", type=int, default=1)
 ap.add_argument("--precision", type=int, default=32)
+ap.add_argument("--lib", default="", help="load this libnbody_b200.so instead of the in-tree build (A/B runs)")
 a = ap.parse_args()
+if a.lib:  # an older build may lack later entry points: bind only what it exports
+    import ctypes
+    from paper_conf_sc_casselldahg24_b200 import _capi
+    from paper_conf_sc_casselldahg24_b200 import build as B
+    B.LIB = os.path.abspath(a.lib)
+    _probe = ctypes.CDLL(B.LIB)
+    for _name in list(_capi.SIGNATURES):
+        if not hasattr(_probe, _name):
+            del _capi.SIGNATURES[_name]
+    _capi.load(build_if_needed=False)  # never rebuild the A/B library from the current sources
+from paper_conf_sc_casselldahg24_b200 import NBody  # noqa: E402
+from workloads import generate  # noqa: E402
+
 pos, vel, mass = generate(a.workload, a.n, a.seed)
 sim = NBody(a.n, a.theta, 1e-3, 1e-3, key_bits=a.key_bits, use_graph=False, traversal=a.traversal,
             multipole=a.multipole, precision=a.precision)
