@@ -421,6 +421,18 @@ nbody_status alloc_f64(nbody_ctx* c) {
   return NBODY_OK;
 }
 
+// S1 fused into K7: valid when one rank updates every body
+// (fp32 mode); the bbox partials are then always those of the current
+// state: set_bodies* computes them after packing, K7 after updating, and a
+// force-only pass only permutes the bodies (min/max of the same set).
+bool bbox_fused(const nbody_ctx* c) {
+  bool comm = false;
+#ifdef NBODY_WITH_NCCL
+  comm = c->comm != nullptr;
+#endif
+  return !c->f64 && c->world == 1 && !c->xpeer && !comm;
+}
+
 // NEXT-3(i) is active: peer exchange over G > 1 ranks with balance on.
 bool balanced(const nbody_ctx* c) { return c->balance && c->xpeer && c->world > 1; }
 
@@ -460,10 +472,12 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     launch_bbox_partial_f64(c->pm64[0], n, c->bbox_part64, c->nbbox, s);
     launch_bbox_final_f64(c->bbox_part64, c->nbbox, c->b, c->grid, s);
   } else {
-    launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
+    // S1: the partials come from the previous K7 (or the packing of
+    // set_bodies) on one rank; ranks that update a slice re-read all bodies
+    if (!bbox_fused(c)) launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);
     launch_bbox_final(c->bbox_part, c->nbbox, c->b, c->grid, s);
   }
-  int front_kernels = 2;
+  int front_kernels = f64 || !bbox_fused(c) ? 2 : 1;
   if (resort) {
     CK(cudaMemsetAsync(c->sort.ghist, 0, sizeof(uint32_t) * 8 * 256, s));
     c->sort.hist_ready = true;  // the key kernel fills the sort's digit histograms
@@ -569,6 +583,8 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
   } else if (integrate && f64) {
     launch_leapfrog_f64(c->pm64[1] + ob, c->vi64[1] + ob, c->acc64, oe - ob, c->dt, c->pm64[0] + ob,
                         c->vi64[0] + ob, s);
+  } else if (integrate && bbox_fused(c)) {  // K7 + the next pass's S1 partials (one rank, all bodies)
+    launch_leapfrog_bbox(c->pm[1], c->vi[1], c->acc, n, float(c->dt), c->pm[0], c->vi[0], c->bbox_part, c->nbbox, s);
   } else if (integrate) {
     launch_leapfrog(c->pm[1] + ob, c->vi[1] + ob, c->acc, oe - ob, float(c->dt), c->pm[0] + ob, c->vi[0] + ob, s);
 #ifdef NBODY_WITH_NCCL
@@ -960,6 +976,7 @@ nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, 
   }
   CK(cudaMemsetAsync(c->bad, 0, sizeof(int), s));
   launch_pack_bodies(dp, dv, dm, n, c->pm[0], c->vi[0], c->bad, s);
+  launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);  // S1 partials of the new state
   CK(cudaGetLastError());
   int bad = 0;
   CK(cudaMemcpyAsync(&bad, c->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
@@ -1012,6 +1029,7 @@ nbody_status nbody_set_bodies_async(nbody_ctx* c, const float* pos, const float*
   CK(cudaEventRecord(c->ev_in_copied[k], c->cstream));
   CK(cudaStreamWaitEvent(c->stream, c->ev_in_copied[k], 0));
   launch_pack_bodies(in, in + 3 * n, in + 6 * n, c->n, c->pm[0], c->vi[0], c->bad_async, c->stream);
+  launch_bbox_partial(c->pm[0], c->n, c->bbox_part, c->nbbox, c->stream);  // S1 partials of the new state
   CK(cudaGetLastError());
   CK(cudaEventRecord(c->ev_in_used[k], c->stream));
   c->ev_in_used_rec[k] = true;

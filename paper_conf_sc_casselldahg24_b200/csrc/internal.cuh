@@ -203,6 +203,9 @@ void launch_direct(const float4* pm, const float4* vi, int64_t n, const int64_t*
 void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt, float4* pm_out,
                      float4* vi_out, cudaStream_t s);
 void launch_fill_float2(float2* p, int64_t count, float2 v, cudaStream_t s);
+// K7 with the next pass's S1 partials fused (partial[6 * nparts], nparts blocks)
+void launch_leapfrog_bbox(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt,
+                          float4* pm_out, float4* vi_out, float* partial, int nparts, cudaStream_t s);
 void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
                         int* bad, cudaStream_t s);
 // out[id][3] <- src[slot].xyz for slots [0, n); id from vi[slot].w

@@ -376,6 +376,26 @@ __device__ __forceinline__ void store_result(const ForceParams& P, int64_t tb, i
   }
 }
 
+// The same for variant 0, from 32-bit quantities that stay live anyway:
+// idx = k - tb (this lane's owned index), k0u = the warp's first slot.
+template <class AccT>
+__device__ __forceinline__ void store_result_idx(const ForceParams& P, uint32_t idx, uint32_t k0u, bool active,
+                                                 const AccT& a, int lane) {
+  if (active) {
+    if constexpr (sizeof(a.x) == 8)
+      P.acc64[idx] = make_double4(a.x, a.y, a.z, 0.0);
+    else
+      P.acc[idx] = make_float4(a.x, a.y, a.z, 0.f);
+    P.count[idx] = a.n;
+  }
+  const uint32_t tot = __reduce_add_sync(kFull, active ? a.n : 0u);
+  if (lane == 0) {
+    atomicAdd(P.total, (unsigned long long)tot);
+    if (P.part)  // NEXT-3(i): this group's cost, to every rank
+      for (int q = 0; q < P.xp.G; ++q) P.xp.gcost[q][k0u >> 5] = tot;
+  }
+}
+
 // ------------------------------------------------------------ variant 1 ----
 constexpr int kV1Warps = 8;
 
@@ -883,7 +903,8 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // so the lists are the ones the walk from the root produces).
   // super-groups are aligned to absolute slots (the same lists on any
   // partition into ranks, hence results bit-identical to one GPU)
-  const uint32_t sgi = kSG > 0 ? uint32_t(k0 / kSG - tb / kSG) : 0u;
+  // (k0 / kSG - tb / kSG, in 32-bit arithmetic: tb mod kSG plus the warp's offset)
+  const uint32_t sgi = kSG > 0 ? (uint32_t(tb) % uint32_t(kSG) + uint32_t(k0 - tb)) / uint32_t(kSG) : 0u;
   int n_acc = -1;
   {
     int2 sgc = make_int2(-1, -1);
@@ -1029,7 +1050,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   while (true) {
     if (na == 0 && S.sg_next < S.sg_nfr) {  // refill the box stack from the super-group frontier
       const int next = S.sg_next;
-      const int take = min(S.sg_nfr - next, kCapA - 64);
+      const int take = min(S.sg_nfr - next, kCapA - 32);  // after a 32-node pop, room for 64 pushes
       const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
       for (int i = lane; i < take; i += 32) S.astk[i] = __ldg(fl + i);
       __syncwarp();

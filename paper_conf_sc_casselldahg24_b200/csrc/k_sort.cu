@@ -31,7 +31,10 @@ namespace {
 #endif
 constexpr int kThreads = NBODY_SORT_THREADS;  // >= 256 (one thread per digit)
 constexpr int kWarps = kThreads / 32;
-constexpr int kItems = 8;
+#ifndef NBODY_SORT_ITEMS
+#define NBODY_SORT_ITEMS 8
+#endif
+constexpr int kItems = NBODY_SORT_ITEMS;
 constexpr int kTile = kThreads * kItems;
 constexpr int kRadix = 256;
 constexpr uint32_t kFlagAgg = 1u << 30;

@@ -2,6 +2,8 @@
 // leapfrog on half-step velocities [A14]: v_{+1/2} = v_{-1/2} + a dt,
 // x_{t+1} = x_t + v_{+1/2} dt (fp32 FMA).  Plus the body packing / id
 // scatter helpers of the C ABI.  All HBM bound, one thread per body.
+#include <cfloat>
+
 #include "internal.cuh"
 
 namespace nb {
@@ -22,6 +24,65 @@ __global__ __launch_bounds__(256) void k_leapfrog(const float4* __restrict__ pm_
   p.z = fmaf(v.z, dt, p.z);
   pm_out[i] = p;
   vi_out[i] = v;
+}
+
+// K7 with S1 of the next step fused: the same update, grid-
+// stride over all n bodies with `gridDim.x` blocks, and each block's min/max
+// of the NEW positions into partial[6 * blockIdx.x ..] -- the bounding-box
+// partials k_bbox_final reduces at the start of the next pass (Alg. 3,
+// P:79-97), so the next pass does not re-read the positions for them.
+// Exact (min/max), hence the same box as k_bbox_partial computes.
+constexpr int kLFThreads = 512;
+
+__device__ __forceinline__ float wmin(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fminf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float wmax(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+__global__ __launch_bounds__(kLFThreads) void k_leapfrog_bbox(const float4* __restrict__ pm_in,
+                                                             const float4* __restrict__ vi_in,
+                                                             const float4* __restrict__ acc, int64_t n, float dt,
+                                                             float4* __restrict__ pm_out, float4* __restrict__ vi_out,
+                                                             float* __restrict__ partial) {
+  float lo0 = FLT_MAX, lo1 = FLT_MAX, lo2 = FLT_MAX;
+  float hi0 = -FLT_MAX, hi1 = -FLT_MAX, hi2 = -FLT_MAX;
+  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+    float4 p = pm_in[i], v = vi_in[i];
+    const float4 a = acc[i];
+    v.x = fmaf(a.x, dt, v.x);
+    v.y = fmaf(a.y, dt, v.y);
+    v.z = fmaf(a.z, dt, v.z);
+    p.x = fmaf(v.x, dt, p.x);
+    p.y = fmaf(v.y, dt, p.y);
+    p.z = fmaf(v.z, dt, p.z);
+    pm_out[i] = p;
+    vi_out[i] = v;
+    lo0 = fminf(lo0, p.x); hi0 = fmaxf(hi0, p.x);
+    lo1 = fminf(lo1, p.y); hi1 = fmaxf(hi1, p.y);
+    lo2 = fminf(lo2, p.z); hi2 = fmaxf(hi2, p.z);
+  }
+  __shared__ float sm[kLFThreads / 32][6];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  lo0 = wmin(lo0); lo1 = wmin(lo1); lo2 = wmin(lo2);
+  hi0 = wmax(hi0); hi1 = wmax(hi1); hi2 = wmax(hi2);
+  if (lane == 0) {
+    sm[w][0] = lo0; sm[w][1] = lo1; sm[w][2] = lo2;
+    sm[w][3] = hi0; sm[w][4] = hi1; sm[w][5] = hi2;
+  }
+  __syncthreads();
+  if (threadIdx.x < 6) {
+    const int c = threadIdx.x;
+    float v = sm[0][c];
+    for (int k = 1; k < kLFThreads / 32; ++k) v = c < 3 ? fminf(v, sm[k][c]) : fmaxf(v, sm[k][c]);
+    partial[6 * blockIdx.x + c] = v;
+  }
 }
 
 // pos[n][3], vel[n][3], mass[n] -> (x, y, z, m), (vx, vy, vz, id bits).
@@ -137,6 +198,12 @@ void launch_leapfrog(const float4* pm_in, const float4* vi_in, const float4* acc
   k_leapfrog<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, n, dt, pm_out, vi_out);
 }
 
+void launch_leapfrog_bbox(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t n, float dt,
+                          float4* pm_out, float4* vi_out, float* partial, int nparts, cudaStream_t s) {
+  if (n <= 0) return;
+  k_leapfrog_bbox<<<unsigned(nparts), kLFThreads, 0, s>>>(pm_in, vi_in, acc, n, dt, pm_out, vi_out, partial);
+}
+
 void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
                         int* bad, cudaStream_t s) {
   k_pack<<<unsigned((n + 255) / 256), 256, 0, s>>>(pos, vel, mass, n, pm, vi, bad);
@@ -183,6 +250,7 @@ void launch_scatter_by_id1_f64(const uint32_t* src, const double4* vi, int64_t n
 void preload_update() {
   touch(k_fill2);
   touch(k_leapfrog);
+  touch(k_leapfrog_bbox);
   touch(k_leapfrog_f64);
   touch(k_pack);
   touch(k_pack_f64);
