@@ -179,14 +179,17 @@ int resolve_bits(int64_t n, int opt) {
 size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
 
 constexpr int kMaxWorld = 256;
-constexpr int64_t kPartPad = 32 * kMaxWorld;  // G * S - N < 32 G
+constexpr int64_t kPartPad = 256 * kMaxWorld;  // G * S - N < 256 G
 
-// [A21] S = ceil(N / G) rounded up to a multiple of 32 (warp groups then
-// coincide with the single-GPU run, so results are bit-identical).
+// [A21] S = ceil(N / G) rounded up to a multiple of kPartUnit = 256 slots:
+// the warp groups (32) and K6a's super-groups (kSG = 256) then coincide
+// with the single-GPU run, so results are bit-identical.
+constexpr int64_t kPartUnit = 256;
+static_assert(kSG <= 0 || kPartUnit % kSG == 0, "rank ranges must start at super-group boundaries");
 void set_part(nbody_ctx* c, int rank, int world) {
   const int64_t n = c->n;
   int64_t s = (n + world - 1) / world;
-  s = (s + 31) / 32 * 32;
+  s = (s + kPartUnit - 1) / kPartUnit * kPartUnit;
   c->rank = rank;
   c->world = world;
   c->own_s = s;
@@ -551,12 +554,13 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     fp.eps2_64 = c->eps * c->eps;
   }
   const bool bal = balanced(c);
-  const int64_t groups = (n + 31) / 32;
-  const int64_t cap_groups = std::min(groups, 2 * ((groups + c->world - 1) / c->world));
+  const int64_t groups = (n + 31) / 32;                      // 32-slot cost groups (one per K6 warp)
+  const int64_t units = (n + kPartUnit - 1) / kPartUnit;      // 256-slot partition units [A21]
+  const int64_t cap_units = std::min(units, 2 * ((units + c->world - 1) / c->world));
   if (bal) {  // NEXT-3(i): the range is read on the device
     fp.part = c->dpart;
     fp.part_rank = c->rank;
-    fp.cap = std::min(n, 32 * cap_groups);
+    fp.cap = std::min(n, kPartUnit * cap_units);
     fp.xp = c->peers;
   }
   int sg_kernels = 0;
@@ -577,7 +581,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
     ++x_kernels;
     if (bal) {  // every group cost has landed: next pass's ranges
-      launch_partition(c->gcost, groups, c->world, n, cap_groups, c->dpart, c->dpart_used, s);
+      launch_partition(c->gcost, groups, c->world, n, cap_units, c->dpart, c->dpart_used, s);
       ++x_kernels;
     }
   } else if (integrate && f64) {
@@ -610,7 +614,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
       launch_xbarrier(c->peers, c->xepoch, 1, c->xerr, s);
       ++x_kernels;
       if (bal) {
-        launch_partition(c->gcost, groups, c->world, n, cap_groups, c->dpart, c->dpart_used, s);
+        launch_partition(c->gcost, groups, c->world, n, cap_units, c->dpart, c->dpart_used, s);
         ++x_kernels;
       }
     }

@@ -167,7 +167,7 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // K6a: the super-group lists of p (p.sg_* must be set); variant-0 K6 reads them.
 void launch_force_sgroups(const ForceParams& p, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
-constexpr int kK6Stats = 46;
+constexpr int kK6Stats = 49;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
@@ -227,10 +227,11 @@ void launch_scatter_by_id1_f64(const uint32_t* src, const double4* vi, int64_t n
 // device and len is only the launch bound (cap).
 void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const float4* acc, int64_t b, int64_t len,
                              float dt, const PeerTable& pt, const int64_t* part, cudaStream_t s);
-// NEXT-3(i): next step's cost-weighted ranges from the group costs of the
-// last pass (identical on every rank): part[0..G] <- boundaries (multiples of
-// 32 slots, each slice <= cap_groups groups); used[0..G] <- the old part.
-void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_groups, int64_t* part,
+// NEXT-3(i): next step's cost-weighted ranges from the 32-slot group costs
+// of the last pass (identical on every rank): part[0..G] <- boundaries
+// (multiples of 256 slots [A21], each slice <= cap_units units of 256);
+// used[0..G] <- the old part.
+void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_units, int64_t* part,
                       int64_t* used, cudaStream_t s);
 // Device-side barrier over the G ranks: signal epoch+1 of `slot` to every
 // rank (release, system scope), then wait until every rank's signal for

@@ -63,15 +63,25 @@ __global__ __launch_bounds__(256) void k_leapfrog_scatter(const float4* __restri
   }
 }
 
-// NEXT-3(i) cost-weighted Hilbert ranges.  Group j (32
-// slots) costs w_j = its interaction count in the last pass (identical data
-// on every rank after the delivery barrier).  With E_j = sum_{i<j} w_i and
-// W = E_J, boundary r is B_r = min{ j : E_j >= ceil(r W / G) }, then clamped
-// in rank order so that every slice has at most cap_groups groups and the
-// remaining ranks can still cover the rest; slot boundary = min(n, 32 B_r).
-// One block: each thread sums a contiguous chunk, a block scan of the chunk
-// sums locates the chunk holding each target, whose thread walks it.
+// NEXT-3(i) cost-weighted Hilbert ranges.  Unit u (256
+// slots = 8 warp groups of 32, the partition unit of [A21]) costs w_u = the
+// interaction count of its slots in the last pass (the sum of its groups'
+// costs; identical data on every rank after the delivery barrier).  With
+// E_u = sum_{i<u} w_i and W = E_U, boundary r is B_r = min{ u : E_u >=
+// ceil(r W / G) }, then clamped in rank order so that every slice has at
+// most cap units and the remaining ranks can still cover the rest; slot
+// boundary = min(n, 256 B_r).  One block: each thread sums a contiguous
+// chunk of units, a block scan of the chunk sums locates the chunk holding
+// each target, whose thread walks it.
 constexpr int kPartThreads = 1024;
+constexpr int kUnitGroups = 8;  // 32-slot cost groups per 256-slot unit
+
+__device__ __forceinline__ unsigned long long unit_cost(const uint32_t* __restrict__ w, int64_t J, int64_t u) {
+  unsigned long long c = 0;
+  const int64_t j1 = min(J, (u + 1) * kUnitGroups);
+  for (int64_t j = u * kUnitGroups; j < j1; ++j) c += w[j];
+  return c;
+}
 
 __global__ __launch_bounds__(kPartThreads) void k_partition(const uint32_t* __restrict__ w, int64_t J, int G,
                                                             int64_t n, int64_t cap, int64_t* __restrict__ part,
@@ -79,10 +89,11 @@ __global__ __launch_bounds__(kPartThreads) void k_partition(const uint32_t* __re
   __shared__ unsigned long long s_pre[kPartThreads + 1];
   __shared__ int64_t s_B[kMaxPeers + 1];
   const int t = threadIdx.x;
-  const int64_t chunk = (J + kPartThreads - 1) / kPartThreads;
-  const int64_t j0 = min(J, int64_t(t) * chunk), j1 = min(J, j0 + chunk);
+  const int64_t U = (J + kUnitGroups - 1) / kUnitGroups;
+  const int64_t chunk = (U + kPartThreads - 1) / kPartThreads;
+  const int64_t u0 = min(U, int64_t(t) * chunk), u1 = min(U, u0 + chunk);
   unsigned long long sum = 0;
-  for (int64_t j = j0; j < j1; ++j) sum += w[j];
+  for (int64_t u = u0; u < u1; ++u) sum += unit_cost(w, J, u);
   s_pre[t + 1] = sum;
   if (t == 0) s_pre[0] = 0;
   __syncthreads();
@@ -101,25 +112,25 @@ __global__ __launch_bounds__(kPartThreads) void k_partition(const uint32_t* __re
       if (t == 0) s_B[r] = 0;
     } else if (s_pre[t] < target && target <= s_pre[t + 1]) {
       unsigned long long e = s_pre[t];
-      int64_t j = j0;
-      while (e < target) e += w[j++];  // E_j >= target first at this j
-      s_B[r] = j;
+      int64_t u = u0;
+      while (e < target) e += unit_cost(w, J, u++);  // E_u >= target first at this u
+      s_B[r] = u;
     }
   }
   __syncthreads();
   if (t == 0) {
     s_B[0] = 0;
-    s_B[G] = J;
+    s_B[G] = U;
     for (int r = 1; r < G; ++r) {
       int64_t b = s_B[r];
       b = max(b, s_B[r - 1]);
       b = min(b, s_B[r - 1] + cap);
-      b = max(b, J - int64_t(G - r) * cap);
+      b = max(b, U - int64_t(G - r) * cap);
       s_B[r] = b;
     }
     for (int r = 0; r <= G; ++r) {
       used[r] = part[r];
-      part[r] = min(n, 32 * s_B[r]);
+      part[r] = min(n, int64_t(kUnitGroups) * 32 * s_B[r]);
     }
   }
 }
@@ -157,9 +168,9 @@ void launch_leapfrog_scatter(const float4* pm_in, const float4* vi_in, const flo
   k_leapfrog_scatter<<<unsigned((len + 255) / 256), 256, 0, s>>>(pm_in, vi_in, acc, b, len, dt, pt, part);
 }
 
-void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_groups, int64_t* part,
+void launch_partition(const uint32_t* gcost, int64_t groups, int G, int64_t n, int64_t cap_units, int64_t* part,
                       int64_t* used, cudaStream_t s) {
-  k_partition<<<1, kPartThreads, 0, s>>>(gcost, groups, G, n, cap_groups, part, used);
+  k_partition<<<1, kPartThreads, 0, s>>>(gcost, groups, G, n, cap_units, part, used);
 }
 
 void launch_xbarrier(const PeerTable& pt, unsigned* epoch, int slot, int* err, cudaStream_t s) {

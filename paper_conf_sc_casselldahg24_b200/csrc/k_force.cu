@@ -894,6 +894,23 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     }
     for (int d = 0; d < 3; ++d) { sb[w2][d] = warp_minf(lo[d]); sb[w2][3 + d] = warp_maxf(hi[d]); }
   }
+  // boxes of the four 8-target quarters of this warp (T pre-test study)
+  float qb[4][6];
+  {
+    const float tx = active ? T.x : inf_stat(), ty = active ? T.y : inf_stat(), tz = active ? T.z : inf_stat();
+    const float ux = active ? T.x : -inf_stat(), uy = active ? T.y : -inf_stat(), uz = active ? T.z : -inf_stat();
+    for (int q = 0; q < 4; ++q) {
+      float v[6] = {tx, ty, tz, ux, uy, uz};
+      for (int d = 0; d < 6; ++d) {
+        float x = v[d];
+        for (int o = 4; o > 0; o >>= 1) {
+          const float y = __shfl_xor_sync(kFull, x, o);
+          x = d < 3 ? fminf(x, y) : fmaxf(x, y);
+        }
+        qb[q][d] = __shfl_sync(kFull, x, 8 * q);
+      }
+    }
+  }
 #endif
   K6STAT(0, 1);
   // Super-group lists (K6a): start from the frontier of this warp's super-
@@ -901,10 +918,9 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // group accepts (every target of this warp then accepts them too, and
   // every frontier node was opened by all of them with all its ancestors,
   // so the lists are the ones the walk from the root produces).
-  // super-groups are aligned to absolute slots (the same lists on any
-  // partition into ranks, hence results bit-identical to one GPU)
-  // (k0 / kSG - tb / kSG, in 32-bit arithmetic: tb mod kSG plus the warp's offset)
-  const uint32_t sgi = kSG > 0 ? (uint32_t(tb) % uint32_t(kSG) + uint32_t(k0 - tb)) / uint32_t(kSG) : 0u;
+  // (rank ranges start at multiples of kSG [A21], so super-groups are the
+  // same absolute slot ranges on any partition: results bit-identical to one GPU)
+  const uint32_t sgi = kSG > 0 ? uint32_t((k0 - tb) / kSG) : 0u;
   int n_acc = -1;
   {
     int2 sgc = make_int2(-1, -1);
@@ -1099,6 +1115,27 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       }
       am &= m;
       rm &= m;
+#ifdef NBODY_K6_STATS
+      {
+        // would the box of the quarters m touches decide this node for all of m?
+        float lo[3] = {inf_stat(), inf_stat(), inf_stat()}, hi[3] = {-inf_stat(), -inf_stat(), -inf_stat()};
+        for (int q = 0; q < 4; ++q)
+          if ((m >> (8 * q)) & 0xffu)
+            for (int d = 0; d < 3; ++d) { lo[d] = fminf(lo[d], qb[q][d]); hi[d] = fmaxf(hi[d], qb[q][3 + d]); }
+        const bool inner = has && g < leaf0;
+        const float2 c = inner ? __ldg(W.rc + g) : make_float2(0.f, 0.f);
+        const float ax0 = lo[0] - r.x, ax1 = r.x - hi[0], ay0 = lo[1] - r.y, ay1 = r.y - hi[1];
+        const float az0 = lo[2] - r.z, az1 = r.z - hi[2];
+        const float mx = fmaxf(0.f, fmaxf(ax0, ax1)), my = fmaxf(0.f, fmaxf(ay0, ay1)), mz = fmaxf(0.f, fmaxf(az0, az1));
+        const float Mx = fmaxf(fabsf(ax0), fabsf(ax1)), My = fmaxf(fabsf(ay0), fabsf(ay1)), Mz = fmaxf(fabsf(az0), fabsf(az1));
+        const float bmin2 = fmaf(mz, mz, fmaf(my, my, mx * mx)), bmax2 = fmaf(Mz, Mz, fmaf(My, My, Mx * Mx));
+        const bool dec = inner && (bmin2 * (1.f - 4e-6f) > c.y || bmax2 * (1.f + 4e-6f) < c.x);
+        K6STAT(46, __reduce_add_sync(kFull, dec ? 1u : 0u));
+        K6STAT(47, __reduce_add_sync(kFull, inner ? 1u : 0u));
+        // batches in which every internal node would be decided
+        K6STAT(48, __all_sync(kFull, dec || !inner) ? 1u : 0u);
+      }
+#endif
       uint32_t und = m & ~(am | rm);
       K6STAT(9, __reduce_add_sync(kFull, __popc(und)));
       K6STAT(16, __reduce_add_sync(kFull, has && (((m & 0xffu) == m) || ((m & 0xff00u) == m) ||
@@ -1301,13 +1338,13 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   int64_t tb, te;
   owned_range(P, tb, te);
-  // list j of this rank: the super-group of absolute slots [g0, g0 + kSG),
-  // g0 = (tb / kSG + j) kSG, boxed over all its bodies (every rank holds the
-  // whole state) so that any partition sees the same lists as one GPU
+  // list j of this rank: slots [tb + j kSG, tb + (j + 1) kSG) -- rank ranges
+  // start at multiples of kSG [A21], so these are the same absolute super-
+  // groups (hence the same lists) on any partition
   const int64_t sgi = int64_t(blockIdx.x) * kSGWarps + w;
-  const int64_t g0 = (tb / kSG + sgi) * kSG;
+  const int64_t g0 = tb + sgi * kSG;
   if (g0 >= te) return;
-  const int64_t g1 = g0 + kSG < int64_t(P.t.n) ? g0 + kSG : int64_t(P.t.n);
+  const int64_t g1 = g0 + kSG < te ? g0 + kSG : te;
   const float inf = __int_as_float(0x7f800000);
   float lx = inf, ly = inf, lz = inf, hx = -inf, hy = -inf, hz = -inf;
   for (int64_t k = g0 + lane; k < g1; k += 32) {
@@ -1403,7 +1440,7 @@ void launch_force_sgroups(const ForceParams& p, cudaStream_t s) {
   if (kSG <= 0 || !p.sg_cnt) return;
   const int64_t nt = p.part ? p.cap : p.t_end - p.t_begin;
   if (nt <= 0) return;
-  const int64_t groups = (nt + kSG - 1) / kSG + 1;  // a range may straddle one more super-group
+  const int64_t groups = (nt + kSG - 1) / kSG;
   const unsigned grid = unsigned((groups + kSGWarps - 1) / kSGWarps);
   if (p.t.rec64)
     k_force_sgroups<true><<<grid, 32 * kSGWarps, 0, s>>>(p);

@@ -29,7 +29,7 @@ def _worker(rank, world, port):
     try:
         from paper_conf_sc_casselldahg24_b200 import dist as D
 
-        # 1. the partition tiles [0, N) with 32-aligned slices
+        # 1. the partition tiles [0, N) with 256-aligned slices [A21]
         for n in (1, 31, 32, 33, 1000, 4097, 10_000_000, 100_000_000):
             mine = D.owned_range(n, rank, world)
             ranges = [None] * world
@@ -37,7 +37,7 @@ def _worker(rank, world, port):
             assert ranges[0][0] == 0 and ranges[-1][1] == n
             for (b0, e0), (b1, e1) in zip(ranges, ranges[1:]):
                 assert e0 == b1 and b0 <= e0
-            assert all((e - b) % 32 == 0 for b, e in ranges[:-1] if e < n)
+            assert all(b % 256 == 0 and (e - b) % 256 == 0 for b, e in ranges[:-1] if e < n)
 
         # 2. every rank gets rank 0's NCCL unique id
         uid = D.broadcast_unique_id(rank)

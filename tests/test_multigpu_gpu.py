@@ -134,28 +134,29 @@ def test_peer_exchange_is_bit_identical(NB, world, n, kw):
 
 
 def _expected_bounds(counts_by_slot, world):
-    """NEXT-3(i) rule (k_exchange.cu k_partition), restated in numpy: group j
-    (32 slots) costs the sum of its slots' interaction counts; boundary r is
-    the first j with E_j = sum_{i<j} w_i >= ceil(r W / G), clamped so that no
-    slice exceeds 2 ceil(J / G) groups; slot boundary min(n, 32 B_r)."""
+    """NEXT-3(i) rule (k_exchange.cu k_partition), restated in numpy: unit u
+    (256 slots, [A21]) costs the sum of its slots' interaction counts;
+    boundary r is the first u with E_u = sum_{i<u} w_i >= ceil(r W / G),
+    clamped so that no slice exceeds 2 ceil(U / G) units; slot boundary
+    min(n, 256 B_r)."""
     n = len(counts_by_slot)
-    J = (n + 31) // 32
-    w = np.zeros(J * 32, np.int64)
+    U = (n + 255) // 256
+    w = np.zeros(U * 256, np.int64)
     w[:n] = counts_by_slot
-    w = w.reshape(J, 32).sum(1)
+    w = w.reshape(U, 256).sum(1)
     E = np.concatenate([[0], np.cumsum(w)])
     W = int(E[-1])
-    cap = min(J, 2 * ((J + world - 1) // world))
+    cap = min(U, 2 * ((U + world - 1) // world))
     B = [0]
     for r in range(1, world):
         t = -(-W * r // world)
         b = int(np.searchsorted(E, t, side="left")) if t > 0 else 0
         b = max(b, B[-1])
         b = min(b, B[-1] + cap)
-        b = max(b, J - (world - r) * cap)
+        b = max(b, U - (world - r) * cap)
         B.append(b)
-    B.append(J)
-    return [min(n, 32 * b) for b in B]
+    B.append(U)
+    return [min(n, 256 * b) for b in B]
 
 
 @pytest.mark.parametrize("world,workload", [(2, "clustered"), (4, "disks"), (8, "clustered")])
@@ -184,7 +185,7 @@ def test_balanced_ranges_follow_last_pass_costs(NB, world, workload):
         got = [s.partition()[2:] for s in ranks]
         assert all(got[r][1] == got[r + 1][0] for r in range(world - 1))
         assert got[0][0] == 0 and got[-1][1] == n
-        assert all(b % 32 == 0 for b, _ in got)
+        assert all(b % 256 == 0 for b, _ in got)
         if prev_counts is None:
             assert got == eq                      # the first pass uses the equal slices
         else:
