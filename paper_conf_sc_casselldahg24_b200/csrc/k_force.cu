@@ -488,6 +488,9 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_SMEM_TOP
 #define NBODY_SMEM_TOP 0
 #endif
+#ifndef NBODY_PMASK_BIT
+#define NBODY_PMASK_BIT 0
+#endif
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 128
 #endif
@@ -752,13 +755,23 @@ __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Targe
     const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
     float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
     uint32_t cnt = 0;
+#if NBODY_PMASK_BIT
+    const uint32_t lbit = 1u << lane;
+#endif
 #pragma unroll kPUnroll
     for (int p = 0; p < (np + 1) >> 1; ++p) {
       const RecPair s = S.prec[p];
       const uint2 mk = *reinterpret_cast<const uint2*>(&S.pmsk[2 * p]);
+#if NBODY_PMASK_BIT  // design variant: test against the lane's bit, predicated count
+      const bool on0 = (mk.x & lbit) != 0u, on1 = (mk.y & lbit) != 0u;
+      interact2<kSoft>(ax, ay, az, s, make_float2(on0 ? s.m.x : 0.f, on1 ? s.m.y : 0.f), nx, ny, nz, e2);
+      if (on0) ++cnt;
+      if (on1) ++cnt;
+#else
       const bool on0 = (mk.x >> lane) & 1u, on1 = (mk.y >> lane) & 1u;
       interact2<kSoft>(ax, ay, az, s, make_float2(on0 ? s.m.x : 0.f, on1 ? s.m.y : 0.f), nx, ny, nz, e2);
       cnt += uint32_t(on0) + uint32_t(on1);
+#endif
     }
     a.x += ax.x + ax.y;
     a.y += ay.x + ay.y;
