@@ -65,7 +65,7 @@ def parse():
                     help="32: fp32 state and interactions (default); 64: the paper's FP64 throughout (NEXT-2)")
     ap.add_argument("--sort-every", type=int, default=1,
                     help="ablation: tree reuse, re-sort every k-th step (NEXT-3(iii)); 1 = Alg. 6")
-    ap.add_argument("--repeats", type=int, default=3, help="timed repeats of K steps (median reported)")
+    ap.add_argument("--repeats", type=int, default=5, help="timed repeats of K steps (median reported, SURVEY 8(d))")
     ap.add_argument("--key-bits", type=int, default=16, help="Hilbert grid bits per axis (0 = paper count rule)")
     ap.add_argument("--no-extras", action="store_true",
                     help="skip the extra blocks of the default run (FP64 mode, config 2, all-pairs calibration)")

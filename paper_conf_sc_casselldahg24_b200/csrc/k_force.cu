@@ -938,6 +938,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   {
     int2 sgc = make_int2(-1, -1);
     if (kSG > 0 && P.sg_cnt) sgc = P.sg_cnt[sgi];
+    K6STAT(49, sgc.x < 0 ? 1u : 0u);  // super-group lists overflowed: this warp walks from the root
     n_acc = sgc.x;
     if (lane == 0) {
       if (sgc.x < 0) S.astk[0] = 1u;
