@@ -12,6 +12,8 @@
 #include <new>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/nbody.h"
 #include "internal.cuh"
 
@@ -468,7 +470,17 @@ void drop_graph(nbody_ctx* c) {
 nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool debug, bool resort = true) {
   const int64_t n = c->n;
   const bool tm = c->timing && s == c->stream;
-  auto mark = [&](int i) -> cudaError_t { return tm ? cudaEventRecord(c->ev[i], s) : cudaSuccess; };
+  // stage boundaries: CUDA events (NBODY_OPT_TIMING, graphs off) and NVTX
+  // ranges around each stage's enqueue (the paper's per-component times,
+  // P:298; host-side, so they bracket the launches with graphs off and
+  // the capture with graphs on)
+  static const char* const kStage[5] = {"S1-S2 bbox + Hilbert keys", "S3 radix sort", "S4-S5 permute + build",
+                                        "S6 force (K6a + K6)", "S7 update (+ exchange)"};
+  auto mark = [&](int i) -> cudaError_t {
+    if (i > 0) nvtxRangePop();
+    if (i < 5) nvtxRangePushA(kStage[i]);
+    return tm ? cudaEventRecord(c->ev[i], s) : cudaSuccess;
+  };
   CK(mark(0));
   const bool f64 = c->f64;
   if (f64) {  // NEXT-2: fp64 bodies
@@ -1068,6 +1080,8 @@ nbody_status nbody_get_positions_async(nbody_ctx* c, float* out) {
 }
 
 nbody_status nbody_compute_accel(nbody_ctx* c) {
+  nvtxRangePushA("nbody_compute_accel");
+  struct Pop { ~Pop() { nvtxRangePop(); } } pop_;
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
   nbody_status s = enqueue_pass(c, c->stream, false, true);
@@ -1078,7 +1092,13 @@ nbody_status nbody_compute_accel(nbody_ctx* c) {
   return NBODY_OK;
 }
 
+struct NvtxScope {
+  explicit NvtxScope(const char* name) { nvtxRangePushA(name); }
+  ~NvtxScope() { nvtxRangePop(); }
+};
+
 nbody_status nbody_step(nbody_ctx* c, int nsteps) {
+  NvtxScope nv("nbody_step");
   CHECK_CTX(c);
   if (!c->loaded) return fail(c, NBODY_ESTATE, "no bodies loaded");
   if (nsteps < 0) return fail(c, NBODY_EINVAL, "nsteps < 0");

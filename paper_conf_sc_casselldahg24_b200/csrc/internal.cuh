@@ -167,7 +167,7 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 // K6a: the super-group lists of p (p.sg_* must be set); variant-0 K6 reads them.
 void launch_force_sgroups(const ForceParams& p, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
-constexpr int kK6Stats = 50;
+constexpr int kK6Stats = 52;
 int force_stats(unsigned long long* out, int n);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------

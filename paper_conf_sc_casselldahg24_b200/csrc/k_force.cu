@@ -491,6 +491,9 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_PMASK_BIT
 #define NBODY_PMASK_BIT 0
 #endif
+#ifndef NBODY_T2BOX
+#define NBODY_T2BOX 0
+#endif
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 128
 #endif
@@ -1144,6 +1147,8 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
         const float Mx = fmaxf(fabsf(ax0), fabsf(ax1)), My = fmaxf(fabsf(ay0), fabsf(ay1)), Mz = fmaxf(fabsf(az0), fabsf(az1));
         const float bmin2 = fmaf(mz, mz, fmaf(my, my, mx * mx)), bmax2 = fmaf(Mz, Mz, fmaf(My, My, Mx * Mx));
         const bool dec = inner && (bmin2 * (1.f - 4e-6f) > c.y || bmax2 * (1.f + 4e-6f) < c.x);
+        K6STAT(50, __reduce_add_sync(kFull, inner && m == amask ? 1u : 0u));
+        K6STAT(51, __reduce_add_sync(kFull, inner && m == amask && rm == m ? 1u : 0u));
         K6STAT(46, __reduce_add_sync(kFull, dec ? 1u : 0u));
         K6STAT(47, __reduce_add_sync(kFull, inner ? 1u : 0u));
         // batches in which every internal node would be decided
@@ -1207,9 +1212,25 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       const bool room = nt + 64 <= S.kT;
       const bool push = rm != 0u && room;
 #endif
-      const uint32_t b1 = __ballot_sync(kFull, push);
-      const uint32_t b2 = __ballot_sync(kFull, push && two);
-      if (push) {
+#if NBODY_T2BOX
+      // design variant: children of a node every active target opened go
+      // back to the box phase (its invariant holds for them), which may
+      // decide them for the whole warp at box-test cost
+      const bool tobox = push && rm == amask && na + 64 <= kCapA;
+      const uint32_t c1 = __ballot_sync(kFull, tobox), c2 = __ballot_sync(kFull, tobox && two);
+      if (tobox) {
+        const int pos = na + __popc(c1 & lt) + __popc(c2 & lt);
+        S.astk[pos] = 2u * g;
+        if (two) S.astk[pos + 1] = 2u * g + 1u;
+      }
+      na += __popc(c1) + __popc(c2);
+      const bool pusht = push && !tobox;
+#else
+      const bool pusht = push;
+#endif
+      const uint32_t b1 = __ballot_sync(kFull, pusht);
+      const uint32_t b2 = __ballot_sync(kFull, pusht && two);
+      if (pusht) {
         const int pos = nt + __popc(b1 & lt) + __popc(b2 & lt);
         S.tstk[pos] = make_uint2(2u * g, rm);
         if (two) S.tstk[pos + 1] = make_uint2(2u * g + 1u, rm);

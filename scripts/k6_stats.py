@@ -19,7 +19,7 @@ kStatNames = ["warps", "A batches", "A nodes", "T batches", "T nodes", "full ent
               "T nodes 1-quarter", "T nodes 1-half", "T mask lanes", "partial q-incid", "partial 1-quarter",
               "partial h-incid", "part sum max q", "part sum max h", "T accept lanes", "T open lanes",
               "part max 8grp", "part max 16grp", "part max lane", "T leaf nodes", "T level-1 nodes", "T internal uniform",
-              "partial popc 1", "partial popc 2", "partial popc <=4", "partial popc <=8", "A guard handovers", "Q-local max-quarter", "H-local max-half", "general partial", "A nodes decided by 128-box", "A nodes decided by 256-box", "A nodes accepted by 128-box", "A internal nodes", "A internal accepted (warp)", "A expanded (warp)", "T internal decided by quarter-union box", "T internal nodes", "T batches all decided", "warps without super-group lists"]
+              "partial popc 1", "partial popc 2", "partial popc <=4", "partial popc <=8", "A guard handovers", "Q-local max-quarter", "H-local max-half", "general partial", "A nodes decided by 128-box", "A nodes decided by 256-box", "A nodes accepted by 128-box", "A internal nodes", "A internal accepted (warp)", "A expanded (warp)", "T internal decided by quarter-union box", "T internal nodes", "T batches all decided", "warps without super-group lists", "T internal full-mask", "T internal full-mask all-open"]
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--workload", default="disks")
@@ -42,12 +42,12 @@ L = _capi.load(build_if_needed=False)
 pos, vel, mass = generate(a.workload, a.n, a.seed)
 sim = NBody(a.n, a.theta, 1e-3, 1e-3, key_bits=16, use_graph=False)
 sim.set_bodies(pos, vel, mass)
-buf = (C.c_uint64 * 50)()
-L.nbody_debug_force_stats(buf, 50)
+buf = (C.c_uint64 * 52)()
+L.nbody_debug_force_stats(buf, 52)
 sim.compute_accel()
 sim.sync()
-got = L.nbody_debug_force_stats(buf, 50)
-assert got == 50, "library not built with NBODY_K6_STATS"
+got = L.nbody_debug_force_stats(buf, 52)
+assert got == 52, "library not built with NBODY_K6_STATS"
 v = list(buf)
 inter = int(sim.get_interactions().sum())
 w = v[0]

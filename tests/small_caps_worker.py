@@ -26,13 +26,13 @@ out = []
 for name, n, seed, theta, quad in [("disks", 40_000, 3, 0.5, False), ("clustered", 30_001, 4, 0.8, False),
                                    ("plummer", 20_000, 5, 0.3, False), ("plummer", 20_000, 6, 0.5, True)]:
     pos, vel, mass = generate(name, n, seed)
-    buf = (C.c_uint64 * 50)()
-    lib.nbody_debug_force_stats(buf, 50)  # reset the counters
+    buf = (C.c_uint64 * 52)()
+    lib.nbody_debug_force_stats(buf, 52)  # reset the counters
     sim = NBody(n, theta, 1e-3, 1e-3, key_bits=16, use_graph=False, multipole=2 if quad else 1)
     sim.set_bodies(pos, vel, mass)
     sim.compute_accel()
     sim.sync()
-    got = lib.nbody_debug_force_stats(buf, 50)
+    got = lib.nbody_debug_force_stats(buf, 52)
     ref = O.step(pos, vel, mass, theta=theta, eps=1e-3, dt=1e-3, key_bits=16, integrate=False, quad=quad)
     cnt = sim.get_interactions()[ref.ids]
     e = rel_errors(sim.get_accel()[ref.ids], ref.acc)
