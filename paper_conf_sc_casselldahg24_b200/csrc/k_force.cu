@@ -494,6 +494,12 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_T2BOX
 #define NBODY_T2BOX 0
 #endif
+// Sparse partial entries (at most NBODY_SPARSE target lanes): kept apart as
+// (id, mask) and evaluated per lane after a 32x32 bit transpose, so a lane
+// only iterates over the entries it is in (0 = off).
+#ifndef NBODY_SPARSE
+#define NBODY_SPARSE 0
+#endif
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 128
 #endif
@@ -583,6 +589,9 @@ struct alignas(16) V0Smem {
   using QP = typename std::conditional<kQuad, QuadPair, char>::type;
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
   QP pq[kQuad ? kCapP / 2 : 1];
+  static constexpr bool kSparse = NBODY_SPARSE > 0 && !kQuad && !kF64_;
+  uint32_t sid[kSparse ? 32 : 1];   // sparse partial entries: node / leaf id ...
+  uint32_t smsk[kSparse ? 32 : 1];  // ... and target mask
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -598,6 +607,19 @@ __device__ __forceinline__ float warp_maxf(float v) {
 
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 __device__ __forceinline__ float inf_stat() { return __int_as_float(0x7f800000); }
+
+// 32x32 bit-matrix transpose across the warp: lane j holds row j on entry;
+// on exit bit j of lane t's word = bit t of lane j's input.
+__device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
+#pragma unroll
+  for (int sh = 16; sh >= 1; sh >>= 1) {
+    const uint32_t m = sh == 16 ? 0x0000ffffu : sh == 8 ? 0x00ff00ffu : sh == 4 ? 0x0f0f0f0fu : sh == 2 ? 0x33333333u
+                                                                                                    : 0x55555555u;
+    const uint32_t y = __shfl_xor_sync(kFull, x, sh);
+    x = (lane & sh) ? ((x & ~m) | ((y & ~m) >> sh)) : ((x & m) | ((y & m) << sh));
+  }
+  return x;
+}
 
 // Transposed-phase filter of the fp64 opening test.
 // With g the group reference point (fp32), c~ = com64 - g, x~ = x - g (exact
@@ -893,6 +915,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   }
 
   int na = 1, nt = 0, nf = 0, np = 0;
+  int ns = 0;  // sparse partial entries staged (NBODY_SPARSE)
 #ifdef NBODY_K6_STATS
   unsigned long long st[kK6Stats] = {};
   int sq[4] = {0, 0, 0, 0}, sh[2] = {0, 0}, s8[8] = {}, s16[16] = {}, s32 = 0;
@@ -956,9 +979,42 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // active lane interacts with it.
   // active lane interacts with it.  id: the node (quadrupole source), 0 for a body.
   // g: the node id (FP64 mode reads its fp64 record rec64[g]).
+  // Sparse entries: each lane walks only the entries it is in (ids in
+  // S.sid, records re-read from the tree), after transposing the masks.
+  auto flush_sparse = [&]() {
+    if constexpr (V0Smem<kQuad, kF64>::kSparse) {
+      __syncwarp();
+      uint32_t wb = transpose32(lane < ns ? S.smsk[lane] : 0u, lane);
+      a.n += __popc(wb);
+      while (__any_sync(kFull, wb != 0u)) {
+        const bool on = wb != 0u;
+        const int j = on ? __ffs(int(wb)) - 1 : 0;
+        wb &= wb - 1u;
+        const float4 r = __ldg(W.rec + S.sid[j]);
+        const Probe pr = probe(r, T);
+        a.add(on, pr.dx, pr.dy, pr.dz, pr.d2, r.w, T.eps2);
+      }
+      ns = 0;
+      __syncwarp();
+    }
+  };
   auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id, uint32_t g) {
     const bool full = want && msk == amask;
-    const bool part = want && msk != amask;
+    bool part = want && msk != amask;
+    if constexpr (V0Smem<kQuad, kF64>::kSparse) {
+      const bool sp = part && __popc(msk) <= NBODY_SPARSE;
+      const uint32_t bs = __ballot_sync(kFull, sp);
+      if (bs) {
+        if (ns + __popc(bs) > 32) flush_sparse();
+        if (sp) {
+          const int pos = ns + __popc(bs & lt);
+          S.sid[pos] = g;
+          S.smsk[pos] = msk;
+        }
+        ns += __popc(bs);
+      }
+      part = part && !sp;
+    }
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
     float4 q0 = make_float4(0.f, 0.f, 0.f, 0.f), q1 = q0;  // NEXT-4: the node's moments (0 for a body)
@@ -1348,6 +1404,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     }
   }
   flush(true);
+  if (ns > 0) flush_sparse();
   store_result(P, tb, k, k0, active, a, lane);
 #ifdef NBODY_K6_STATS
   if (lane == 0)
