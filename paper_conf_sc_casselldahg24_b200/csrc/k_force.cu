@@ -500,6 +500,9 @@ constexpr int kV0Warps = 4;
 #ifndef NBODY_SPARSE
 #define NBODY_SPARSE 0
 #endif
+#ifndef NBODY_SPARSE_REC
+#define NBODY_SPARSE_REC 0  // 1: stage the records in shared memory instead of re-reading them
+#endif
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 128
 #endif
@@ -590,7 +593,11 @@ struct alignas(16) V0Smem {
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
   QP pq[kQuad ? kCapP / 2 : 1];
   static constexpr bool kSparse = NBODY_SPARSE > 0 && !kQuad && !kF64_;
+#if NBODY_SPARSE_REC
+  float4 srec[kSparse ? 32 : 1];    // sparse partial entries: record ...
+#else
   uint32_t sid[kSparse ? 32 : 1];   // sparse partial entries: node / leaf id ...
+#endif
   uint32_t smsk[kSparse ? 32 : 1];  // ... and target mask
 };
 
@@ -990,7 +997,11 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
         const bool on = wb != 0u;
         const int j = on ? __ffs(int(wb)) - 1 : 0;
         wb &= wb - 1u;
+#if NBODY_SPARSE_REC
+        const float4 r = S.srec[j];
+#else
         const float4 r = __ldg(W.rec + S.sid[j]);
+#endif
         const Probe pr = probe(r, T);
         a.add(on, pr.dx, pr.dy, pr.dz, pr.d2, r.w, T.eps2);
       }
@@ -1008,7 +1019,11 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
         if (ns + __popc(bs) > 32) flush_sparse();
         if (sp) {
           const int pos = ns + __popc(bs & lt);
+#if NBODY_SPARSE_REC
+          S.srec[pos] = r;
+#else
           S.sid[pos] = g;
+#endif
           S.smsk[pos] = msk;
         }
         ns += __popc(bs);
