@@ -475,7 +475,10 @@ __global__ __launch_bounds__(kV2Threads) void k_force_skiplist(const ForceParams
 }
 
 // ------------------------------------------------------------ variant 0 ----
-constexpr int kV0Warps = 4;
+#ifndef NBODY_V0_WARPS
+#define NBODY_V0_WARPS 4
+#endif
+constexpr int kV0Warps = NBODY_V0_WARPS;
 // Sized for 8 blocks x 4 warps per SM (26.4 KB shared memory per block);
 // stack overflow is handled (box phase: hand over as MIXED; transposed
 // phase: per-lane mask walk), so the capacities only affect speed.
