@@ -397,7 +397,8 @@ nbody_status allocate(nbody_ctx* c) {
   c->sort.tiles = tiles;
   c->sort.ghist = (uint32_t*)sortmem;
   c->sort.tile_ctr = c->sort.ghist + 8 * 256;
-  c->sort.status = c->sort.tile_ctr + 8;
+  c->sort.gpre = c->sort.tile_ctr + 8;
+  c->sort.status = c->sort.gpre + 8 * 256;
   return NBODY_OK;
 }
 
@@ -513,7 +514,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
       launch_permute_f64(c->pm64[0], c->vi64[0], c->idx[c->perm_buf], n, c->pm64[1], c->vi64[1], s);
     else
       launch_permute(c->pm[0], c->vi[0], c->idx[c->perm_buf], n, c->pm[1], c->vi[1], s);
-    front_kernels += 1 + c->sort.passes + 1;
+    front_kernels += 1 + 1 + c->sort.passes + 1;  // keys, digit prefix, sort passes, permute
   } else {
     // tree reuse (NEXT-3(iii), [A23]): keep the current (previous Hilbert)
     // order; the leaves are the current state

@@ -142,6 +142,7 @@ struct SortPlan {
   uint32_t* ghist;    // [8][256]
   uint32_t* status;   // [passes][tiles][256]
   uint32_t* tile_ctr; // [8]
+  uint32_t* gpre;     // [8][256] exclusive prefix of ghist per pass (k_hist_prefix)
   bool hist_ready;    // ghist already filled (by the key kernel)
 };
 int64_t sort_tiles(int64_t n);

@@ -21,7 +21,10 @@ namespace nb {
 namespace {
 
 constexpr int kAPThreads = 256;
-constexpr int kAPT = 2;                   // targets per thread
+#ifndef NBODY_AP_T
+#define NBODY_AP_T 2
+#endif
+constexpr int kAPT = NBODY_AP_T;           // targets per thread
 constexpr int kAPTile = 2048;             // sources per shared-memory tile (32 KB)
 constexpr int kAPPairs = kAPTile / 2;
 

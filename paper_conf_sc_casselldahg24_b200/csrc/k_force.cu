@@ -479,14 +479,16 @@ __global__ __launch_bounds__(kV2Threads) void k_force_skiplist(const ForceParams
 #define NBODY_V0_WARPS 4
 #endif
 constexpr int kV0Warps = NBODY_V0_WARPS;
-// Sized for 8 blocks x 4 warps per SM (26.4 KB shared memory per block);
-// stack overflow is handled (box phase: hand over as MIXED; transposed
-// phase: per-lane mask walk), so the capacities only affect speed.
+// Sized for 6 blocks x 4 warps per SM: 80 registers per thread and 31 KB of
+// shared memory per block (round 2: 6 blocks with these lists beat 8 blocks
+// at 64 registers by 3.7 %, profiles/r02_ab_k6.md); stack overflow is
+// handled (box phase: hand over as MIXED; transposed phase: per-lane mask
+// walk; K6a frontier: refilled in chunks), so the capacities only affect speed.
 #ifndef NBODY_CAP_T
-#define NBODY_CAP_T 288
+#define NBODY_CAP_T 256
 #endif
 #ifndef NBODY_V0_MINB
-#define NBODY_V0_MINB 8
+#define NBODY_V0_MINB 6
 #endif
 #ifndef NBODY_SMEM_TOP
 #define NBODY_SMEM_TOP 0
@@ -507,7 +509,7 @@ constexpr int kV0Warps = NBODY_V0_WARPS;
 #define NBODY_SPARSE_REC 0  // 1: stage the records in shared memory instead of re-reading them
 #endif
 #ifndef NBODY_CAP_A
-#define NBODY_CAP_A 128
+#define NBODY_CAP_A 320
 #endif
 constexpr int kCapA = NBODY_CAP_A;  // box-phase stack (ids)
 constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
@@ -515,7 +517,7 @@ constexpr int kCapT = NBODY_CAP_T;  // transposed-phase stack (id, mask)
 #define NBODY_CAP_F 96
 #endif
 #ifndef NBODY_CAP_P
-#define NBODY_CAP_P 64
+#define NBODY_CAP_P 96
 #endif
 #ifndef NBODY_FUNROLL
 #define NBODY_FUNROLL 2
@@ -541,7 +543,17 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 #ifndef NBODY_QCAP_T
 #define NBODY_QCAP_T 224
 #endif
+#ifndef NBODY_QCAP_A
+#define NBODY_QCAP_A 128
+#endif
 template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad ? NBODY_QCAP_F : kF64 ? 64 : kCapF; }
+// box-phase stack: the quadrupole and FP64 variants keep a smaller one (their
+// larger records leave less shared memory)
+template <bool kQuad, bool kF64> constexpr int cap_a() { return kQuad || kF64 ? NBODY_QCAP_A : kCapA; }
+#ifndef NBODY_QCAP_P
+#define NBODY_QCAP_P 64
+#endif
+template <bool kQuad, bool kF64> constexpr int cap_p() { return kQuad || kF64 ? NBODY_QCAP_P : kCapP; }
 template <bool kQuad, bool kF64> constexpr int cap_t() { return kQuad ? NBODY_QCAP_T : kF64 ? 192 : kCapT; }
 
 // Records in pairs, component-interleaved, so that one 16-B shared load
@@ -585,23 +597,27 @@ struct alignas(16) V0Smem {
   double4 tpos64[kF64 ? 32 : 1];  // NEXT-2 FP64 mode: exact target positions
   static constexpr int kF = cap_f<kQuad, kF64_>(), kT = cap_t<kQuad, kF64_>();
   RecPair frec[kF64 ? 1 : kF / 2];  // monopole / body records, all lanes
-  RecPair prec[kF64 ? 1 : kCapP / 2];  // monopole / body records, ...
+  static constexpr int kP = cap_p<kQuad, kF64_>();
+  RecPair prec[kF64 ? 1 : kP / 2];  // monopole / body records, ...
   double4 frec64[kF64 ? kF : 1];    // NEXT-2 FP64 mode: the same lists in fp64
-  double4 prec64[kF64 ? kCapP : 1];
-  uint32_t pmsk[kCapP];     // ... for the lanes in the mask
-  uint32_t astk[kCapA];
+  double4 prec64[kF64 ? kP : 1];
+  uint32_t pmsk[kP];        // ... for the lanes in the mask
+  static constexpr int kA = cap_a<kQuad, kF64_>();
+  uint32_t astk[kA];
   uint2 tstk[kT];     // (id, mask of the targets that reached it)
   int sg_next, sg_nfr;  // super-group frontier: next entry, length (K6a)
   using QP = typename std::conditional<kQuad, QuadPair, char>::type;
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
-  QP pq[kQuad ? kCapP / 2 : 1];
+  QP pq[kQuad ? kP / 2 : 1];
   static constexpr bool kSparse = NBODY_SPARSE > 0 && !kQuad && !kF64_;
+#if NBODY_SPARSE > 0
 #if NBODY_SPARSE_REC
   float4 srec[kSparse ? 32 : 1];    // sparse partial entries: record ...
 #else
   uint32_t sid[kSparse ? 32 : 1];   // sparse partial entries: node / leaf id ...
 #endif
   uint32_t smsk[kSparse ? 32 : 1];  // ... and target mask
+#endif
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -992,6 +1008,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // Sparse entries: each lane walks only the entries it is in (ids in
   // S.sid, records re-read from the tree), after transposing the masks.
   auto flush_sparse = [&]() {
+#if NBODY_SPARSE > 0
     if constexpr (V0Smem<kQuad, kF64>::kSparse) {
       __syncwarp();
       uint32_t wb = transpose32(lane < ns ? S.smsk[lane] : 0u, lane);
@@ -1011,10 +1028,12 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       ns = 0;
       __syncwarp();
     }
+#endif
   };
   auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id, uint32_t g) {
     const bool full = want && msk == amask;
     bool part = want && msk != amask;
+#if NBODY_SPARSE > 0
     if constexpr (V0Smem<kQuad, kF64>::kSparse) {
       const bool sp = part && __popc(msk) <= NBODY_SPARSE;
       const uint32_t bs = __ballot_sync(kFull, sp);
@@ -1033,6 +1052,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       }
       part = part && !sp;
     }
+#endif
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
     float4 q0 = make_float4(0.f, 0.f, 0.f, 0.f), q1 = q0;  // NEXT-4: the node's moments (0 for a body)
@@ -1114,7 +1134,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       K6STAT(11, (nf + 1) >> 1);
       nf = 0;
     }
-    if (np > kCapP - 32 || (all && np > 0)) {
+    if (np > S.kP - 32 || (all && np > 0)) {
       if constexpr (kF64)
         dense_part64<kSoft>(S, np, T, a, lane);
       else
@@ -1157,7 +1177,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   while (true) {
     if (na == 0 && S.sg_next < S.sg_nfr) {  // refill the box stack from the super-group frontier
       const int next = S.sg_next;
-      const int take = min(S.sg_nfr - next, kCapA - 32);  // after a 32-node pop, room for 64 pushes
+      const int take = min(S.sg_nfr - next, S.kA - 32);  // after a 32-node pop, room for 64 pushes
       const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
       for (int i = lane; i < take; i += 32) S.astk[i] = __ldg(fl + i);
       __syncwarp();
@@ -1290,7 +1310,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       // design variant: children of a node every active target opened go
       // back to the box phase (its invariant holds for them), which may
       // decide them for the whole warp at box-test cost
-      const bool tobox = push && rm == amask && na + 64 <= kCapA;
+      const bool tobox = push && rm == amask && na + 64 <= S.kA;
       const uint32_t c1 = __ballot_sync(kFull, tobox), c2 = __ballot_sync(kFull, tobox && two);
       if (tobox) {
         const int pos = na + __popc(c1 & lt) + __popc(c2 & lt);
@@ -1333,7 +1353,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       const uint32_t g = has ? S.astk[base + lane] : 0u;
       __syncwarp();
       na = base;
-      const bool guard = na + 64 > kCapA;
+      const bool guard = na + 64 > S.kA;
       int cls = 0;  // 1 dense, 2 expand, 3 transposed
 #ifdef NBODY_K6_STATS
       bool guard_open = false;

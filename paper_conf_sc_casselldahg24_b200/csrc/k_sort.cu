@@ -81,6 +81,26 @@ __global__ __launch_bounds__(kThreads) void k_hist(const K* __restrict__ keys, i
     if (sh[i]) atomicAdd(&ghist[i], sh[i]);
 }
 
+// The global digit offsets of every pass, once per sort: gpre[p][d] =
+// sum_{d' < d} ghist[p][d'] (one block; thread d, a loop over the passes).
+__global__ __launch_bounds__(kRadix) void k_hist_prefix(const uint32_t* __restrict__ ghist, int passes,
+                                                        uint32_t* __restrict__ gpre) {
+  __shared__ uint32_t s[kRadix];
+  const int d = threadIdx.x;
+  for (int p = 0; p < passes; ++p) {
+    s[d] = ghist[p * kRadix + d];
+    __syncthreads();
+    for (int o = 1; o < kRadix; o <<= 1) {  // inclusive scan
+      const uint32_t v = d >= o ? s[d - o] : 0u;
+      __syncthreads();
+      s[d] += v;
+      __syncthreads();
+    }
+    gpre[p * kRadix + d] = s[d] - ghist[p * kRadix + d];
+    __syncthreads();
+  }
+}
+
 // Exclusive scan of v over threads 0..255 (others pass 0); every thread of
 // the block must call.  Returns the exclusive prefix for the caller.
 __device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t* s_tmp) {
@@ -178,7 +198,7 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
     }
   }
   const uint32_t dl = scan256(tid < kRadix ? cnt : 0u, s_tmp);
-  const uint32_t gb = scan256(tid < kRadix ? ghist[tid] : 0u, s_tmp);
+  const uint32_t gb = tid < kRadix ? ghist[tid] : 0u;  // this pass's global digit offsets (k_hist_prefix)
   // Publish this tile's digit counts first (successors may look back past
   // it), then place the keys in tile-local digit order in shared memory: that
   // needs only local offsets, and it frees the key registers for the look-back.
@@ -277,13 +297,14 @@ void run_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s
     const int hb = int(p.tiles < 4 * kNumSMs ? p.tiles : int64_t(4 * kNumSMs));
     k_hist<K><<<hb, kThreads, 0, s>>>(static_cast<const K*>(keys[0]), p.n, p.passes, p.ghist);
   }
+  k_hist_prefix<<<1, kRadix, 0, s>>>(p.ghist, p.passes, p.gpre);
   for (int pass = 0; pass < p.passes; ++pass) {
     const int in = pass & 1, out = in ^ 1;
     const K* kin = static_cast<const K*>(keys[in]);
     K* kout = static_cast<K*>(keys[out]);
     const bool first = pass == 0, last = pass == p.passes - 1;
     uint32_t* st = p.status + size_t(pass) * size_t(p.tiles) * kRadix;
-    const uint32_t* gh = p.ghist + pass * kRadix;
+    const uint32_t* gh = p.gpre + pass * kRadix;  // exclusive prefix (the kernel's `ghist` argument)
     const unsigned grid = unsigned(p.tiles);
     const size_t sm = dyn_smem<K>();
     if (first && last)
@@ -306,7 +327,7 @@ void run_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s
 int64_t sort_tiles(int64_t n) { return (n + kTile - 1) / kTile; }
 
 size_t sort_scratch_bytes(int64_t n) {
-  return sizeof(uint32_t) * (8 * kRadix + 8 + size_t(8) * size_t(sort_tiles(n)) * kRadix);
+  return sizeof(uint32_t) * (8 * kRadix + 8 + 8 * kRadix + size_t(8) * size_t(sort_tiles(n)) * kRadix);
 }
 
 int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaStream_t s) {
@@ -321,6 +342,7 @@ int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaSt
 // Load every kernel of this file now (see preload_all in capi.cu).
 void preload_sort() {
   touch(k_hist<uint32_t>);
+  touch(k_hist_prefix);
   touch(k_hist<unsigned long long>);
   touch(k_onesweep<uint32_t, false, false>);
   touch(k_onesweep<uint32_t, false, true>);

@@ -20,7 +20,7 @@ for tool in memcheck racecheck synccheck initcheck; do
 done
 # small capacities: spill walks and the box guard on every warp
 lib=/tmp/libnbody_smallcaps_san.so
-NBODY_NVCC_FLAGS="-DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 -DNBODY_CAP_A=64 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64" \
+NBODY_NVCC_FLAGS="-DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 -DNBODY_CAP_A=64 -DNBODY_QCAP_A=64 -DNBODY_QCAP_P=32 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64" \
   python -c "from paper_conf_sc_casselldahg24_b200 import build as B; B.LIB='$lib'; B.build(force=True)"
 for tool in memcheck racecheck; do
   log=gpurun_out/${tag}_sanitizer_${tool}_smallcaps.log

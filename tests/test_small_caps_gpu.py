@@ -31,7 +31,7 @@ def test_overflow_paths_match_the_oracle(tmp_path):
     lib = str(tmp_path / "libnbody_smallcaps.so")
     env = dict(os.environ)
     env["NBODY_NVCC_FLAGS"] = ("-DNBODY_K6_STATS -DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 "
-                               "-DNBODY_CAP_A=64 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64")
+                               "-DNBODY_CAP_A=64 -DNBODY_QCAP_A=64 -DNBODY_QCAP_P=32 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64")
     code = f"from paper_conf_sc_casselldahg24_b200 import build as B; B.LIB = {lib!r}; B.build(force=True)"
     subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=os.path.dirname(HERE))
     env["NBODY_TEST_LIB"] = lib
