@@ -493,21 +493,7 @@ constexpr int kV0Warps = NBODY_V0_WARPS;
 #ifndef NBODY_SMEM_TOP
 #define NBODY_SMEM_TOP 0
 #endif
-#ifndef NBODY_PMASK_BIT
-#define NBODY_PMASK_BIT 0
-#endif
-#ifndef NBODY_T2BOX
-#define NBODY_T2BOX 0
-#endif
-// Sparse partial entries (at most NBODY_SPARSE target lanes): kept apart as
-// (id, mask) and evaluated per lane after a 32x32 bit transpose, so a lane
-// only iterates over the entries it is in (0 = off).
-#ifndef NBODY_SPARSE
-#define NBODY_SPARSE 0
-#endif
-#ifndef NBODY_SPARSE_REC
-#define NBODY_SPARSE_REC 0  // 1: stage the records in shared memory instead of re-reading them
-#endif
+
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 320
 #endif
@@ -549,11 +535,19 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad ? NBODY_QCAP_F : kF64 ? 64 : kCapF; }
 // box-phase stack: the quadrupole and FP64 variants keep a smaller one (their
 // larger records leave less shared memory)
-template <bool kQuad, bool kF64> constexpr int cap_a() { return kQuad || kF64 ? NBODY_QCAP_A : kCapA; }
+#ifndef NBODY_F64CAP_A
+#define NBODY_F64CAP_A 128
+#endif
+template <bool kQuad, bool kF64> constexpr int cap_a() {
+  return kQuad ? NBODY_QCAP_A : kF64 ? NBODY_F64CAP_A : kCapA;
+}
 #ifndef NBODY_QCAP_P
 #define NBODY_QCAP_P 64
 #endif
-template <bool kQuad, bool kF64> constexpr int cap_p() { return kQuad || kF64 ? NBODY_QCAP_P : kCapP; }
+#ifndef NBODY_F64CAP_P
+#define NBODY_F64CAP_P 64
+#endif
+template <bool kQuad, bool kF64> constexpr int cap_p() { return kQuad ? NBODY_QCAP_P : kF64 ? NBODY_F64CAP_P : kCapP; }
 template <bool kQuad, bool kF64> constexpr int cap_t() { return kQuad ? NBODY_QCAP_T : kF64 ? 192 : kCapT; }
 
 // Records in pairs, component-interleaved, so that one 16-B shared load
@@ -609,15 +603,6 @@ struct alignas(16) V0Smem {
   using QP = typename std::conditional<kQuad, QuadPair, char>::type;
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
   QP pq[kQuad ? kP / 2 : 1];
-  static constexpr bool kSparse = NBODY_SPARSE > 0 && !kQuad && !kF64_;
-#if NBODY_SPARSE > 0
-#if NBODY_SPARSE_REC
-  float4 srec[kSparse ? 32 : 1];    // sparse partial entries: record ...
-#else
-  uint32_t sid[kSparse ? 32 : 1];   // sparse partial entries: node / leaf id ...
-#endif
-  uint32_t smsk[kSparse ? 32 : 1];  // ... and target mask
-#endif
 };
 
 __device__ __forceinline__ float warp_minf(float v) {
@@ -634,18 +619,6 @@ __device__ __forceinline__ float warp_maxf(float v) {
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 __device__ __forceinline__ float inf_stat() { return __int_as_float(0x7f800000); }
 
-// 32x32 bit-matrix transpose across the warp: lane j holds row j on entry;
-// on exit bit j of lane t's word = bit t of lane j's input.
-__device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
-#pragma unroll
-  for (int sh = 16; sh >= 1; sh >>= 1) {
-    const uint32_t m = sh == 16 ? 0x0000ffffu : sh == 8 ? 0x00ff00ffu : sh == 4 ? 0x0f0f0f0fu : sh == 2 ? 0x33333333u
-                                                                                                    : 0x55555555u;
-    const uint32_t y = __shfl_xor_sync(kFull, x, sh);
-    x = (lane & sh) ? ((x & ~m) | ((y & ~m) >> sh)) : ((x & m) | ((y & m) << sh));
-  }
-  return x;
-}
 
 // Transposed-phase filter of the fp64 opening test.
 // With g the group reference point (fp32), c~ = com64 - g, x~ = x - g (exact
@@ -806,23 +779,13 @@ __device__ __forceinline__ void dense_part(V0Smem<kQuad>& S, int np, const Targe
     const float2 nx = f2(-T.x), ny = f2(-T.y), nz = f2(-T.z), e2 = f2(T.eps2);
     float2 ax = f2(0.f), ay = f2(0.f), az = f2(0.f);
     uint32_t cnt = 0;
-#if NBODY_PMASK_BIT
-    const uint32_t lbit = 1u << lane;
-#endif
 #pragma unroll kPUnroll
     for (int p = 0; p < (np + 1) >> 1; ++p) {
       const RecPair s = S.prec[p];
       const uint2 mk = *reinterpret_cast<const uint2*>(&S.pmsk[2 * p]);
-#if NBODY_PMASK_BIT  // design variant: test against the lane's bit, predicated count
-      const bool on0 = (mk.x & lbit) != 0u, on1 = (mk.y & lbit) != 0u;
-      interact2<kSoft>(ax, ay, az, s, make_float2(on0 ? s.m.x : 0.f, on1 ? s.m.y : 0.f), nx, ny, nz, e2);
-      if (on0) ++cnt;
-      if (on1) ++cnt;
-#else
       const bool on0 = (mk.x >> lane) & 1u, on1 = (mk.y >> lane) & 1u;
       interact2<kSoft>(ax, ay, az, s, make_float2(on0 ? s.m.x : 0.f, on1 ? s.m.y : 0.f), nx, ny, nz, e2);
       cnt += uint32_t(on0) + uint32_t(on1);
-#endif
     }
     a.x += ax.x + ax.y;
     a.y += ay.x + ay.y;
@@ -941,7 +904,6 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   }
 
   int na = 1, nt = 0, nf = 0, np = 0;
-  int ns = 0;  // sparse partial entries staged (NBODY_SPARSE)
 #ifdef NBODY_K6_STATS
   unsigned long long st[kK6Stats] = {};
   int sq[4] = {0, 0, 0, 0}, sh[2] = {0, 0}, s8[8] = {}, s16[16] = {}, s32 = 0;
@@ -1005,54 +967,9 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   // active lane interacts with it.
   // active lane interacts with it.  id: the node (quadrupole source), 0 for a body.
   // g: the node id (FP64 mode reads its fp64 record rec64[g]).
-  // Sparse entries: each lane walks only the entries it is in (ids in
-  // S.sid, records re-read from the tree), after transposing the masks.
-  auto flush_sparse = [&]() {
-#if NBODY_SPARSE > 0
-    if constexpr (V0Smem<kQuad, kF64>::kSparse) {
-      __syncwarp();
-      uint32_t wb = transpose32(lane < ns ? S.smsk[lane] : 0u, lane);
-      a.n += __popc(wb);
-      while (__any_sync(kFull, wb != 0u)) {
-        const bool on = wb != 0u;
-        const int j = on ? __ffs(int(wb)) - 1 : 0;
-        wb &= wb - 1u;
-#if NBODY_SPARSE_REC
-        const float4 r = S.srec[j];
-#else
-        const float4 r = __ldg(W.rec + S.sid[j]);
-#endif
-        const Probe pr = probe(r, T);
-        a.add(on, pr.dx, pr.dy, pr.dz, pr.d2, r.w, T.eps2);
-      }
-      ns = 0;
-      __syncwarp();
-    }
-#endif
-  };
   auto append = [&](bool want, const float4& r, uint32_t msk, uint32_t id, uint32_t g) {
     const bool full = want && msk == amask;
-    bool part = want && msk != amask;
-#if NBODY_SPARSE > 0
-    if constexpr (V0Smem<kQuad, kF64>::kSparse) {
-      const bool sp = part && __popc(msk) <= NBODY_SPARSE;
-      const uint32_t bs = __ballot_sync(kFull, sp);
-      if (bs) {
-        if (ns + __popc(bs) > 32) flush_sparse();
-        if (sp) {
-          const int pos = ns + __popc(bs & lt);
-#if NBODY_SPARSE_REC
-          S.srec[pos] = r;
-#else
-          S.sid[pos] = g;
-#endif
-          S.smsk[pos] = msk;
-        }
-        ns += __popc(bs);
-      }
-      part = part && !sp;
-    }
-#endif
+    const bool part = want && msk != amask;
     const uint32_t bf = __ballot_sync(kFull, full);
     const uint32_t bp = __ballot_sync(kFull, part);
     float4 q0 = make_float4(0.f, 0.f, 0.f, 0.f), q1 = q0;  // NEXT-4: the node's moments (0 for a body)
@@ -1306,25 +1223,9 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       const bool room = nt + 64 <= S.kT;
       const bool push = rm != 0u && room;
 #endif
-#if NBODY_T2BOX
-      // design variant: children of a node every active target opened go
-      // back to the box phase (its invariant holds for them), which may
-      // decide them for the whole warp at box-test cost
-      const bool tobox = push && rm == amask && na + 64 <= S.kA;
-      const uint32_t c1 = __ballot_sync(kFull, tobox), c2 = __ballot_sync(kFull, tobox && two);
-      if (tobox) {
-        const int pos = na + __popc(c1 & lt) + __popc(c2 & lt);
-        S.astk[pos] = 2u * g;
-        if (two) S.astk[pos + 1] = 2u * g + 1u;
-      }
-      na += __popc(c1) + __popc(c2);
-      const bool pusht = push && !tobox;
-#else
-      const bool pusht = push;
-#endif
-      const uint32_t b1 = __ballot_sync(kFull, pusht);
-      const uint32_t b2 = __ballot_sync(kFull, pusht && two);
-      if (pusht) {
+      const uint32_t b1 = __ballot_sync(kFull, push);
+      const uint32_t b2 = __ballot_sync(kFull, push && two);
+      if (push) {
         const int pos = nt + __popc(b1 & lt) + __popc(b2 & lt);
         S.tstk[pos] = make_uint2(2u * g, rm);
         if (two) S.tstk[pos + 1] = make_uint2(2u * g + 1u, rm);
@@ -1442,7 +1343,6 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     }
   }
   flush(true);
-  if (ns > 0) flush_sparse();
   store_result(P, tb, k, k0, active, a, lane);
 #ifdef NBODY_K6_STATS
   if (lane == 0)
