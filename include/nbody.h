@@ -128,6 +128,11 @@ typedef struct {
   float ms_force;             /*  K1+K2, K3, K4+K5, K6, K7                */
   float ms_update;
   int kernels_per_step;       /* library kernel launches in one step      */
+  float lane_util;            /* K6 dense-phase lane utilisation (interacting
+                                 lanes / 32 per list slot) since the counters
+                                 were last read by nbody_debug_force_stats, in
+                                 a -DNBODY_K6_STATS build; -1 otherwise (the
+                                 product build carries no counters)        */
 } nbody_stats;
 
 /* Library version (major*10000 + minor*100 + patch). */

@@ -47,7 +47,7 @@ class nbody_stats(C.Structure):
     _fields_ = [("n", C.c_int64), ("key_bits", C.c_int), ("levels", C.c_int), ("steps", C.c_int64),
                 ("interactions", C.c_uint64), ("ms_bbox_keys", C.c_float), ("ms_sort", C.c_float),
                 ("ms_build", C.c_float), ("ms_force", C.c_float), ("ms_update", C.c_float),
-                ("kernels_per_step", C.c_int)]
+                ("kernels_per_step", C.c_int), ("lane_util", C.c_float)]
 
 
 _P = C.c_void_p

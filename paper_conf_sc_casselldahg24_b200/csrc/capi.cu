@@ -1639,6 +1639,17 @@ nbody_status nbody_get_stats(nbody_ctx* c, nbody_stats* out) {
     out->interactions = t;
   }
   out->kernels_per_step = c->kernels_per_step;
+  // lane utilisation of K6's dense phase, from the design counters
+  // (NBODY_K6_STATS builds only; counters since the last reset): interacting
+  // lanes / (32 x dense-list slots)
+  out->lane_util = -1.f;
+  {
+    unsigned long long st[9];
+    if (force_stats(st, 9, false) == 9) {
+      const double slots = 32.0 * double(st[5] + st[6]);
+      if (slots > 0) out->lane_util = float(double(st[7] + st[8]) / slots);
+    }
+  }
   if (c->ev_valid) {
     CK(cudaEventSynchronize(c->ev[5]));
     float* dst[5] = {&out->ms_bbox_keys, &out->ms_sort, &out->ms_build, &out->ms_force, &out->ms_update};

@@ -169,7 +169,7 @@ void launch_force(const ForceParams& p, int variant, cudaStream_t s);
 void launch_force_sgroups(const ForceParams& p, cudaStream_t s);
 // K6 event counters (NBODY_K6_STATS builds; else returns 0); reading resets them
 constexpr int kK6Stats = 52;
-int force_stats(unsigned long long* out, int n);
+int force_stats(unsigned long long* out, int n, bool reset = true);
 
 // ---- NEXT-1: all-pairs direct sum for sampled targets (fp64) ----------------
 // Lazy module loading (the CUDA 12 default) loads a kernel at its first

@@ -64,14 +64,15 @@ __device__ unsigned long long g_k6_stats[kK6Stats];
 #define K6STAT(i, v) ((void)0)
 #endif
 
-int force_stats(unsigned long long* out, int n) {
+int force_stats(unsigned long long* out, int n, bool reset) {
 #ifdef NBODY_K6_STATS
   if (n > kK6Stats) n = kK6Stats;
   if (cudaMemcpyFromSymbol(out, g_k6_stats, sizeof(unsigned long long) * n) != cudaSuccess) return -1;
   static const unsigned long long zero[kK6Stats] = {};
-  if (cudaMemcpyToSymbol(g_k6_stats, zero, sizeof(zero)) != cudaSuccess) return -1;
+  if (reset && cudaMemcpyToSymbol(g_k6_stats, zero, sizeof(zero)) != cudaSuccess) return -1;
   return n;
 #else
+  (void)reset;
   (void)out;
   (void)n;
   return 0;

@@ -32,13 +32,14 @@ for name, n, seed, theta, quad in [("disks", 40_000, 3, 0.5, False), ("clustered
     sim.set_bodies(pos, vel, mass)
     sim.compute_accel()
     sim.sync()
+    lane_util = sim.stats()["lane_util"]  # peeks at the counters (no reset)
     got = lib.nbody_debug_force_stats(buf, 52)
     ref = O.step(pos, vel, mass, theta=theta, eps=1e-3, dt=1e-3, key_bits=16, integrate=False, quad=quad)
     cnt = sim.get_interactions()[ref.ids]
     e = rel_errors(sim.get_accel()[ref.ids], ref.acc)
     out.append({"case": f"{name} n={n} theta={theta} quad={quad}", "stats_len": got,
                 "spill_walks": int(buf[14]), "guard_handovers": int(buf[36]),
-                "counts_equal": bool((cnt == ref.count).all()),
+                "counts_equal": bool((cnt == ref.count).all()), "lane_util": lane_util,
                 "rms": float(np.sqrt(np.mean(e ** 2))), "max": float(e.max())})
     sim.close()
 print(json.dumps(out))

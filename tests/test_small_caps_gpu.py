@@ -39,8 +39,15 @@ def test_overflow_paths_match_the_oracle(tmp_path):
                        capture_output=True, text=True)
     res = json.loads(r.stdout.strip().splitlines()[-1])
     assert B.LIB != lib  # the product library of this process is untouched
+    from paper_conf_sc_casselldahg24_b200 import NBody
+    from workloads import generate
+    sim = NBody(2000)
+    sim.set_bodies(*generate("plummer", 2000, 1))
+    sim.compute_accel()
+    assert sim.stats()["lane_util"] == -1.0  # the product build carries no counters
     for c in res:
         assert c["stats_len"] == 52, c
         assert c["spill_walks"] > 0 and c["guard_handovers"] > 0, c
         assert c["counts_equal"], c
+        assert 0.0 < c["lane_util"] <= 1.0, c  # nbody_get_stats reports the counters of a stats build
         assert c["rms"] <= ACC_RMS_TOL and c["max"] <= ACC_MAX_TOL, c
