@@ -120,6 +120,15 @@ __device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t* s_tmp) {
   return pre + x - v;
 }
 
+// Design instrumentation (-DNBODY_SORT_PROFILE builds only): SM cycles per
+// phase of a tile, summed over tiles (thread 0's clock at the block barriers).
+#ifdef NBODY_SORT_PROFILE
+__device__ unsigned long long g_sort_prof[8];
+#define SORT_T(i) (tid == 0 ? (tp[i] = clock64()) : 0ll)
+#else
+#define SORT_T(i) 0ll
+#endif
+
 template <class K, bool kFirst, bool kWriteKeys>
 __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                        K* __restrict__ kout, uint32_t* __restrict__ vout, int64_t n,
@@ -133,9 +142,14 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
   __shared__ uint32_t s_tile;
 
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+#ifdef NBODY_SORT_PROFILE
+  long long tp[6];
+#endif
+  SORT_T(0);
   if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
   for (int i = tid; i < kWarps * kRadix; i += kThreads) s_whist[i] = 0;
   __syncthreads();
+  SORT_T(1);
   const int64_t tile = s_tile;
   const int64_t base = tile * kTile;
 
@@ -187,6 +201,7 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
     __syncwarp();
   }
   __syncthreads();
+  SORT_T(2);
 
   // Per digit: exclusive prefix over warps (in place) and the tile count.
   uint32_t cnt = 0;
@@ -208,6 +223,7 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
     mine.store((tile == 0 ? kFlagInc : kFlagAgg) | cnt, cuda::memory_order_relaxed);
   }
   __syncthreads();
+  SORT_T(3);
 #pragma unroll
   for (int i = 0; i < kItems; ++i) {
     if (d[i] < kRadix) {
@@ -256,6 +272,7 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
     }
   }
   __syncthreads();
+  SORT_T(4);
 
   // ... and write runs of consecutive global addresses.
   const int valid = int(n - base < kTile ? n - base : int64_t(kTile));
@@ -266,6 +283,13 @@ __global__ __launch_bounds__(kThreads, NBODY_SORT_MINB) void k_onesweep(const K*
     if (kWriteKeys) kout[g] = key;
     vout[g] = s_vals[j];
   }
+#ifdef NBODY_SORT_PROFILE
+  __syncthreads();
+  SORT_T(5);
+  if (tid == 0)
+    for (int i = 0; i < 5; ++i) atomicAdd(&g_sort_prof[i], (unsigned long long)(tp[i + 1] - tp[i]));
+  if (tid == 0) atomicAdd(&g_sort_prof[5], 1ull);
+#endif
 }
 
 template <class K>
@@ -338,6 +362,15 @@ int launch_radix_sort(const SortPlan& p, void* keys[2], uint32_t* idx[2], cudaSt
   return p.passes & 1;
 }
 
+
+#ifdef NBODY_SORT_PROFILE
+extern "C" int nbody_debug_sort_profile(unsigned long long* out) {  // design builds only (not in nbody.h)
+  if (cudaMemcpyFromSymbol(out, g_sort_prof, sizeof(unsigned long long) * 6) != cudaSuccess) return -1;
+  static const unsigned long long zero[8] = {};
+  cudaMemcpyToSymbol(g_sort_prof, zero, sizeof(zero));
+  return 6;
+}
+#endif
 
 // Load every kernel of this file now (see preload_all in capi.cu).
 void preload_sort() {
