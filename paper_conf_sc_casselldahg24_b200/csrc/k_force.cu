@@ -494,13 +494,6 @@ constexpr int kV0Warps = NBODY_V0_WARPS;
 #ifndef NBODY_SMEM_TOP
 #define NBODY_SMEM_TOP 0
 #endif
-// T pre-test: a (node, mask) entry popped from the T stack is first tested
-// against the box of the target quarters its mask touches; only the entries
-// that box cannot decide for all of the mask go on (second stack) to the
-// per-target test (0 = off).
-#ifndef NBODY_TPRE
-#define NBODY_TPRE 0
-#endif
 
 #ifndef NBODY_CAP_A
 #define NBODY_CAP_A 320
@@ -608,10 +601,6 @@ struct alignas(16) V0Smem {
   uint32_t astk[kA];
   uint2 tstk[kT];     // (id, mask of the targets that reached it)
   int sg_next, sg_nfr;  // super-group frontier: next entry, length (K6a)
-#if NBODY_TPRE
-  float qb[4][6];       // boxes of the four 8-target quarters (lo xyz, hi xyz)
-  uint2 t2stk[64];      // pre-tested entries the quarter boxes left undecided
-#endif
   using QP = typename std::conditional<kQuad, QuadPair, char>::type;
   QP fq[kQuad ? kF / 2 : 1];  // NEXT-4: each entry's second moments (0 for a body), paired
   QP pq[kQuad ? kP / 2 : 1];
@@ -916,25 +905,6 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
   }
 
   int na = 1, nt = 0, nf = 0, np = 0;
-#if NBODY_TPRE
-  int nt2 = 0;
-  {
-    const float tx = active ? T.x : inf, ty = active ? T.y : inf, tz = active ? T.z : inf;
-    const float ux = active ? T.x : -inf, uy = active ? T.y : -inf, uz = active ? T.z : -inf;
-    float v[6] = {tx, ty, tz, ux, uy, uz};
-#pragma unroll
-    for (int d = 0; d < 6; ++d) {
-      float x = v[d];
-#pragma unroll
-      for (int o = 4; o > 0; o >>= 1) {
-        const float y = __shfl_xor_sync(kFull, x, o);
-        x = d < 3 ? fminf(x, y) : fmaxf(x, y);
-      }
-      if ((lane & 7) == 0) S.qb[lane >> 3][d] = x;
-    }
-    __syncwarp();
-  }
-#endif
 #ifdef NBODY_K6_STATS
   unsigned long long st[kK6Stats] = {};
   int sq[4] = {0, 0, 0, 0}, sh[2] = {0, 0}, s8[8] = {}, s16[16] = {}, s32 = 0;
@@ -1132,76 +1102,23 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       if (lane == 0) S.sg_next = next + take;
       na = take;
     }
-#if NBODY_TPRE
-    if (nt >= 32 || nt2 >= 32 || (na == 0 && (nt > 0 || nt2 > 0))) {
-      // pre-test from the T stack, or the per-target test of the entries it
-      // left undecided (full batches first; at the end whatever remains)
-      const bool full_test = nt2 >= 32 || nt == 0;
-      const int avail = full_test ? nt2 : nt;
-#else
     if (nt >= 32 || (na == 0 && nt > 0)) {
-      constexpr bool full_test = true;
-      const int avail = nt;
-#endif
       // ---- T: transposed classification of up to 32 (node, mask) entries
-      const int take = avail < 32 ? avail : 32;
-      const int base = avail - take;
+      const int take = nt < 32 ? nt : 32;
+      const int base = nt - take;
       K6STAT(3, 1);
       K6STAT(4, take);
       K6STAT(15, take < 32);
       const bool has = lane < take;
-#if NBODY_TPRE
-      const uint2 e = has ? (full_test ? S.t2stk[base + lane] : S.tstk[base + lane]) : make_uint2(leaf0, 0u);
-      __syncwarp();
-      if (full_test) nt2 = base; else nt = base;
-#else
       const uint2 e = has ? S.tstk[base + lane] : make_uint2(leaf0, 0u);
       __syncwarp();
       nt = base;
-#endif
       const uint32_t g = e.x, m = e.y;
       const float4 r = __ldg(W.rec + g);
-      uint32_t am = 0u, rm = 0u;
-#if NBODY_TPRE
-      if (!full_test) {
-        // box of the quarters m touches against the node's filter thresholds
-        // (the box phase's bounds, valid for any box holding those targets)
-        bool dec = false;
-        if (has && g < leaf0) {
-          float lo0 = inf, lo1 = inf, lo2 = inf, hi0 = -inf, hi1 = -inf, hi2 = -inf;
-#pragma unroll
-          for (int q = 0; q < 4; ++q)
-            if ((m >> (8 * q)) & 0xffu) {
-              lo0 = fminf(lo0, S.qb[q][0]); lo1 = fminf(lo1, S.qb[q][1]); lo2 = fminf(lo2, S.qb[q][2]);
-              hi0 = fmaxf(hi0, S.qb[q][3]); hi1 = fmaxf(hi1, S.qb[q][4]); hi2 = fmaxf(hi2, S.qb[q][5]);
-            }
-          const float2 c = __ldg(W.rc + g);
-          const float ax0 = lo0 - r.x, ax1 = r.x - hi0, ay0 = lo1 - r.y, ay1 = r.y - hi1;
-          const float az0 = lo2 - r.z, az1 = r.z - hi2;
-          const float nx = fmaxf(0.f, fmaxf(ax0, ax1)), ny = fmaxf(0.f, fmaxf(ay0, ay1)),
-                      nz = fmaxf(0.f, fmaxf(az0, az1));
-          const float fx = fmaxf(fabsf(ax0), fabsf(ax1)), fy = fmaxf(fabsf(ay0), fabsf(ay1)),
-                      fz = fmaxf(fabsf(az0), fabsf(az1));
-          const float dmin2 = fmaf(nz, nz, fmaf(ny, ny, nx * nx));
-          const float dmax2 = fmaf(fz, fz, fmaf(fy, fy, fx * fx));
-          if (dmin2 * (1.f - 4e-6f) > c.y) {
-            am = m;
-            dec = true;
-          } else if (dmax2 * (1.f + 4e-6f) < c.x) {
-            rm = m;
-            dec = true;
-          }
-        }
-        const bool defer = has && !dec;
-        const uint32_t bd = __ballot_sync(kFull, defer);
-        if (defer) S.t2stk[nt2 + __popc(bd & lt)] = e;
-        nt2 += __popc(bd);
-      } else
-#endif
-      {
       float cx = 0.f, cy = 0.f, cz = 0.f;
       float KA = inf, KO = inf;  // leaves: always interact, never open
       if (g < leaf0) tfilter_prep(r, __ldg(tfp + g), gx, gy, gz, kk1, kk0, cx, cy, cz, KA, KO);
+      uint32_t am = 0u, rm = 0u;
       {
         // S = 2 c'.x' - |x'|^2; accept iff S < KA  <=>  S - KA < 0, open iff
         // S > KO  <=>  KO - S < 0: one exact rounding each (a nonzero
@@ -1279,7 +1196,6 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
           } while (und);
         }
       }
-      }  // full per-target test
       if (g >= leaf0 && g - kid0 < 32u) am &= ~(1u << (g - kid0));  // a leaf never acts on itself
       append(am != 0u, r, am, g < leaf0 ? g : 0u, g);
       // children of opened nodes, with the mask of the targets that opened them
