@@ -25,7 +25,14 @@ constexpr int kAPThreads = 256;
 #define NBODY_AP_T 2
 #endif
 constexpr int kAPT = NBODY_AP_T;           // targets per thread
-constexpr int kAPTile = 2048;             // sources per shared-memory tile (32 KB)
+#ifndef NBODY_AP_TILE
+#define NBODY_AP_TILE 2048
+#endif
+#ifndef NBODY_AP_UNROLL
+#define NBODY_AP_UNROLL 8
+#endif
+constexpr int kAPTile = NBODY_AP_TILE;    // sources per shared-memory tile (32 KB at 2048)
+constexpr int kAPUnroll = NBODY_AP_UNROLL;  // #pragma unroll takes no macros
 constexpr int kAPPairs = kAPTile / 2;
 
 struct alignas(16) SrcPair {
@@ -98,7 +105,7 @@ __global__ __launch_bounds__(kAPThreads) void k_allpairs32(const float4* __restr
 #pragma unroll
     for (int i = 0; i < kAPT; ++i) fx[i] = fy[i] = fz[i] = f2(0.f);
     const int np = int(j1 - base >= kAPTile ? kAPPairs : (j1 - base + 1) >> 1);
-#pragma unroll 4
+#pragma unroll kAPUnroll
     for (int p = 0; p < np; ++p) {
       const SrcPair s = sp[p];
 #pragma unroll
