@@ -531,7 +531,7 @@ constexpr int kCapP = NBODY_CAP_P;  // dense list: entries with a lane mask
 #define NBODY_QCAP_T 224
 #endif
 #ifndef NBODY_QCAP_A
-#define NBODY_QCAP_A 128
+#define NBODY_QCAP_A 256
 #endif
 template <bool kQuad, bool kF64> constexpr int cap_f() { return kQuad ? NBODY_QCAP_F : kF64 ? 64 : kCapF; }
 // box-phase stack: the quadrupole and FP64 variants keep a smaller one (their
