@@ -1,6 +1,6 @@
 """Config 4 (clustered Plummer, N = 1e8) sampled parity on one GPU: keys and
 the permutation in full, node records on sampled nodes of all 27 levels,
-forces and counts on sampled targets (scripts/parity_large.py; ~90 s)."""
+forces and counts on sampled targets (tests/parity_large.py; ~90 s)."""
 import os
 import subprocess
 import sys
