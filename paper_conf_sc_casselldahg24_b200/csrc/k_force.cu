@@ -20,6 +20,13 @@
 //
 // Variant 0 (default), group-classified transposed walk.  A warp owns 32
 // Hilbert-consecutive targets with bounding box B.
+//   K6a (k_force_sgroups, a separate kernel launched first): one warp per
+//      super-group of kSG = 256 consecutive targets runs the box phase below
+//      against the super-group's box from the root; the nodes every target
+//      of the super-group accepts go to its `acc` list, the nodes it cannot
+//      decide (and leaves) to its `frontier`.  A variant-0 warp appends `acc`
+//      as full dense entries and starts its own box phase from the frontier
+//      instead of the root (same lists: its box lies inside the super-group's).
 //   A. Box phase (lanes = nodes): lanes classify 32 nodes at a time against B
 //      with exact fp64 bounds of the opening test over all of B: every lane
 //      accepts (-> dense list, all lanes), every lane opens (-> children are
