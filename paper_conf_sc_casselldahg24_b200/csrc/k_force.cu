@@ -625,7 +625,9 @@ __device__ __forceinline__ float warp_maxf(float v) {
 }
 
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
+#ifdef NBODY_K6_STATS
 __device__ __forceinline__ float inf_stat() { return __int_as_float(0x7f800000); }
+#endif
 
 
 // Transposed-phase filter of the fp64 opening test.

@@ -124,9 +124,9 @@ __device__ __forceinline__ uint32_t scan256(uint32_t v, uint32_t* s_tmp) {
 // phase of a tile, summed over tiles (thread 0's clock at the block barriers).
 #ifdef NBODY_SORT_PROFILE
 __device__ unsigned long long g_sort_prof[8];
-#define SORT_T(i) (tid == 0 ? (tp[i] = clock64()) : 0ll)
+#define SORT_T(i) (void)(tid == 0 ? (tp[i] = clock64()) : 0ll)
 #else
-#define SORT_T(i) 0ll
+#define SORT_T(i) ((void)0)
 #endif
 
 template <class K, bool kFirst, bool kWriteKeys>
