@@ -544,7 +544,7 @@ nbody_status enqueue_pass(nbody_ctx* c, cudaStream_t s, bool integrate, bool deb
     build_kernels = c->tree.L;
   } else {
     launch_build_fused(c->tree, c->pm[1], debug, s);
-    build_kernels = c->tree.L < 1 ? 0 : (c->tree.L > 10 ? 2 : 1);
+    build_kernels = build_fused_kernels(c->tree);
   }
   CK(cudaMemsetAsync(c->total, 0, sizeof(unsigned long long), s));
   CK(mark(3));

@@ -157,6 +157,7 @@ void launch_permute(const float4* pm_in, const float4* vi_in, const uint32_t* pe
 void launch_build(const TreeView& t, const float4* leaves, cudaStream_t s);  // level by level (reference)
 // levels 1..10 fused per 1024-leaf subtree + one block for the top levels;
 // keep_all also stores every node's moments/box (debug views)
+int build_fused_kernels(const TreeView& t);  // kernel launches of launch_build_fused
 void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, cudaStream_t s);
 // NEXT-2 FP64 mode: leaves are t.rec64 + 2^L (fp64 bodies); boxes in fp64
 void launch_permute_f64(const double4* pm_in, const double4* vi_in, const uint32_t* perm, int64_t n,

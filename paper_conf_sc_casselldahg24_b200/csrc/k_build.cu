@@ -182,6 +182,9 @@ __global__ __launch_bounds__(256) void k_build_level(TreeView t, int l) {
 // kernels); only the subtree roots (level top) keep moments/boxes in global
 // memory unless keep_all (debug views).
 constexpr int kFuseLevels = 10;
+#ifndef NBODY_UPPER_WIDE
+#define NBODY_UPPER_WIDE 3  // upper levels built by one grid each before the one-block kernel
+#endif
 constexpr int kFuseHalf = 1 << (kFuseLevels - 1);  // level-1 nodes per block
 constexpr int kFuseThreads = 256;
 
@@ -365,7 +368,25 @@ void launch_build_fused(const TreeView& t, const float4* leaves, bool keep_all, 
     k_build_fused<true, false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
   else
     k_build_fused<false, false><<<grid, kFuseThreads, 0, s>>>(t, leaves, top, keep_all);
-  if (t.L > top) k_build_upper<false><<<1, 1024, 0, s>>>(t, top + 1);
+  int from = top + 1;
+#if NBODY_UPPER_WIDE > 0
+  // the widest upper levels (thousands of nodes) one grid each, the narrow
+  // rest in the one-block kernel (same arithmetic, bit-identical records)
+  if (!t.quad)
+    for (; from <= t.L && from <= top + NBODY_UPPER_WIDE; ++from)
+      k_build_level<<<unsigned((t.count[from] + 255) / 256), 256, 0, s>>>(t, from);
+#endif
+  if (t.L >= from) k_build_upper<false><<<1, 1024, 0, s>>>(t, from);
+}
+
+int build_fused_kernels(const TreeView& t) {  // launches of launch_build_fused
+  if (t.L < 1) return 0;
+  const int levels = t.quad ? kFuseLevels - 1 : kFuseLevels;
+  const int top = t.L < levels ? t.L : levels;
+  int from = top + 1, k = 1;
+  if (!t.quad)
+    for (; from <= t.L && from <= top + NBODY_UPPER_WIDE; ++from) ++k;
+  return k + (t.L >= from ? 1 : 0);
 }
 
 void launch_build_fused_f64(const TreeView& t, bool keep_all, cudaStream_t s) {
