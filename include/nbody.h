@@ -248,6 +248,23 @@ nbody_status nbody_get_state(nbody_ctx *ctx, float *pos_m, float *vel_id);
  * NBODY_EINVAL in mode 32 (and nbody_get_state is NBODY_EINVAL in mode 64). */
 nbody_status nbody_get_state64(nbody_ctx *ctx, double *pos_m, double *vel_id);
 
+/* Checkpoint / resume: restore a state exactly as nbody_get_state wrote it
+ * -- pos_m[n][4] = (x, y, z, m), vel_id[n][4] = (vx, vy, vz, id as float
+ * bits), in slot order, host or device (copied) -- and the step counter
+ * `steps` (nbody_stats.steps of the checkpointed context).  Unlike
+ * nbody_set_bodies, the slot order and the ids are kept, so the next sort's
+ * tie order (the stable sort of Alg. 7 P:201-212 by current slot, [A10]) and
+ * the tree-reuse phase (NBODY_OPT_SORT_EVERY, [A23]) are those of the
+ * checkpointed run: stepping a restored context is bit-identical to
+ * stepping the original.  Every rank passes the same arrays.  NBODY_EINVAL
+ * for null pointers, steps < 0, ids that are not a permutation of [0, n),
+ * or invalid values [A18] (the context then holds no bodies); in FP64 mode
+ * use nbody_set_state64. */
+nbody_status nbody_set_state(nbody_ctx *ctx, const float *pos_m, const float *vel_id, int64_t steps);
+/* NEXT-2 FP64 mode: as nbody_set_state with the layout of
+ * nbody_get_state64 (ids as exact integers in fp64).  NBODY_EINVAL in mode 32. */
+nbody_status nbody_set_state64(nbody_ctx *ctx, const double *pos_m, const double *vel_id, int64_t steps);
+
 nbody_status nbody_get_stats(nbody_ctx *ctx, nbody_stats *out);
 
 /* ---- NEXT-1: the paper's All-Pairs baseline, sampled -----------

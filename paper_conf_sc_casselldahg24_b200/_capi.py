@@ -82,6 +82,8 @@ SIGNATURES = {
     "nbody_get_positions64": (_S, [_P, _P]),
     "nbody_get_velocities64": (_S, [_P, _P]),
     "nbody_get_state64": (_S, [_P, _P, _P]),
+    "nbody_set_state": (_S, [_P, _P, _P, _I64]),
+    "nbody_set_state64": (_S, [_P, _P, _P, _I64]),
     "nbody_debug_level64": (_S, [_P, C.c_int, C.POINTER(_I64), _P, _P]),
     "nbody_get_stats": (_S, [_P, C.POINTER(nbody_stats)]),
     "nbody_direct_accel": (_S, [_P, _P, _I64, _P]),

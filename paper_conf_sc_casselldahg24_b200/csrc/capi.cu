@@ -1009,6 +1009,57 @@ nbody_status nbody_set_bodies(nbody_ctx* c, const float* pos, const float* vel, 
   return NBODY_OK;
 }
 
+// Restore a slot-order state written by nbody_get_state(64) (checkpoint /
+// resume): the records go straight into the current-state buffers, so the
+// slot order -- which decides the stable sort's tie order (Alg. 7, [A10]) --
+// and the ids survive, and the step counter restores the tree-reuse phase.
+static nbody_status set_state_common(nbody_ctx* c, const void* pos_m, const void* vel_id, int64_t steps,
+                                     size_t rec) {
+  if (!pos_m || !vel_id) return fail(c, NBODY_EINVAL, "null input");
+  if (steps < 0) return fail(c, NBODY_EINVAL, "steps < 0");
+  const int64_t n = c->n;
+  cudaStream_t s = c->stream;
+  void* pm = c->f64 ? static_cast<void*>(c->pm64[0]) : static_cast<void*>(c->pm[0]);
+  void* vi = c->f64 ? static_cast<void*>(c->vi64[0]) : static_cast<void*>(c->vi[0]);
+  CK(cudaMemcpyAsync(pm, pos_m, rec * size_t(n), cudaMemcpyDefault, s));
+  CK(cudaMemcpyAsync(vi, vel_id, rec * size_t(n), cudaMemcpyDefault, s));
+  CK(cudaMemsetAsync(c->bad, 0, sizeof(int), s));
+  CK(cudaMemsetAsync(c->idx[1], 0, sizeof(uint32_t) * size_t(n), s));  // id claims (the sort rewrites idx)
+  if (c->f64) {
+    launch_check_state_f64(c->pm64[0], c->vi64[0], n, c->idx[1], c->bad, s);
+  } else {
+    launch_check_state(c->pm[0], c->vi[0], n, c->idx[1], c->bad, s);
+    launch_bbox_partial(c->pm[0], n, c->bbox_part, c->nbbox, s);  // S1 partials of the restored state
+  }
+  CK(cudaGetLastError());
+  int bad = 0;
+  CK(cudaMemcpyAsync(&bad, c->bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  c->have_force = false;
+  c->keys_dbg_valid = false;
+  if (bad) {
+    c->loaded = false;
+    return fail(c, NBODY_EINVAL, (bad & 4) ? "state ids are not a permutation of [0, n)"
+                                 : (bad & 2) ? "masses must be finite and > 0"
+                                             : "non-finite position or velocity");
+  }
+  c->loaded = true;
+  c->steps = steps;
+  return NBODY_OK;
+}
+
+nbody_status nbody_set_state(nbody_ctx* c, const float* pos_m, const float* vel_id, int64_t steps) {
+  CHECK_CTX(c);
+  if (c->f64) return fail(c, NBODY_EINVAL, "FP64 mode: use nbody_set_state64");
+  return set_state_common(c, pos_m, vel_id, steps, sizeof(float4));
+}
+
+nbody_status nbody_set_state64(nbody_ctx* c, const double* pos_m, const double* vel_id, int64_t steps) {
+  CHECK_CTX(c);
+  if (!c->f64) return fail(c, NBODY_EINVAL, "nbody_set_state64 needs NBODY_OPT_PRECISION = 64");
+  return set_state_common(c, pos_m, vel_id, steps, sizeof(double4));
+}
+
 // Lazily create the copy stream, events and staging buffers of the
 // pipelined transfers.
 static nbody_status ensure_xfer(nbody_ctx* c) {

@@ -210,6 +210,11 @@ void launch_leapfrog_bbox(const float4* pm_in, const float4* vi_in, const float4
                           float4* pm_out, float4* vi_out, float* partial, int nparts, cudaStream_t s);
 void launch_pack_bodies(const float* pos, const float* vel, const float* mass, int64_t n, float4* pm, float4* vi,
                         int* bad, cudaStream_t s);
+// nbody_set_state: validate a restored state (flags as k_pack, 4 = ids not a
+// permutation of [0, n); seen[n] zeroed by the caller)
+void launch_check_state(const float4* pm, const float4* vi, int64_t n, uint32_t* seen, int* bad, cudaStream_t s);
+void launch_check_state_f64(const double4* pm, const double4* vi, int64_t n, uint32_t* seen, int* bad,
+                            cudaStream_t s);
 // out[id][3] <- src[slot].xyz for slots [0, n); id from vi[slot].w
 void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s);
 void launch_scatter_by_id1(const uint32_t* src, const float4* vi, int64_t n, uint32_t* out, cudaStream_t s);

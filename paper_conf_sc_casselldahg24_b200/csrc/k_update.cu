@@ -104,6 +104,38 @@ __global__ __launch_bounds__(256) void k_pack(const float* __restrict__ pos, con
   vi[i] = make_float4(u, v, w, __int_as_float(int(i)));
 }
 
+// nbody_set_state: validate a restored slot-order state in place (the
+// checks of k_pack [A18], plus: the ids are a permutation of [0, n) --
+// seen[] zeroed by the caller; a second claim of an id is a duplicate).
+template <class V4, class S>
+__device__ __forceinline__ void check_state(const V4& p, const V4& v, uint32_t id, bool id_ok, int64_t n,
+                                            uint32_t* seen, int* bad) {
+  int flag = 0;
+  if (!(isfinite(p.x) && isfinite(p.y) && isfinite(p.z) && isfinite(v.x) && isfinite(v.y) && isfinite(v.z)))
+    flag |= 1;
+  if (!(isfinite(p.w) && p.w > S(0))) flag |= 2;
+  if (!id_ok || int64_t(id) >= n || atomicExch(seen + id, 1u) != 0u) flag |= 4;
+  if (flag) atomicOr(bad, flag);
+}
+
+__global__ __launch_bounds__(256) void k_check_state(const float4* __restrict__ pm, const float4* __restrict__ vi,
+                                                     int64_t n, uint32_t* __restrict__ seen, int* __restrict__ bad) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const float4 v = vi[i];
+  check_state<float4, float>(pm[i], v, uint32_t(__float_as_int(v.w)), true, n, seen, bad);
+}
+
+__global__ __launch_bounds__(256) void k_check_state_f64(const double4* __restrict__ pm,
+                                                         const double4* __restrict__ vi, int64_t n,
+                                                         uint32_t* __restrict__ seen, int* __restrict__ bad) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const double4 v = vi[i];
+  const bool ok = v.w >= 0.0 && v.w < 4294967296.0 && double(uint32_t(v.w)) == v.w;  // an exact integer id
+  check_state<double4, double>(pm[i], v, ok ? uint32_t(v.w) : 0u, ok, n, seen, bad);
+}
+
 __global__ __launch_bounds__(256) void k_scatter3(const float4* __restrict__ src, const float4* __restrict__ vi,
                                                   int64_t n, float* __restrict__ out) {
   const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -209,6 +241,15 @@ void launch_pack_bodies(const float* pos, const float* vel, const float* mass, i
   k_pack<<<unsigned((n + 255) / 256), 256, 0, s>>>(pos, vel, mass, n, pm, vi, bad);
 }
 
+void launch_check_state(const float4* pm, const float4* vi, int64_t n, uint32_t* seen, int* bad, cudaStream_t s) {
+  k_check_state<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm, vi, n, seen, bad);
+}
+
+void launch_check_state_f64(const double4* pm, const double4* vi, int64_t n, uint32_t* seen, int* bad,
+                            cudaStream_t s) {
+  k_check_state_f64<<<unsigned((n + 255) / 256), 256, 0, s>>>(pm, vi, n, seen, bad);
+}
+
 void launch_scatter_by_id3(const float4* src, const float4* vi, int64_t n, float* out, cudaStream_t s) {
   if (n <= 0) return;  // a rank may own no slots
   k_scatter3<<<unsigned((n + 255) / 256), 256, 0, s>>>(src, vi, n, out);
@@ -254,6 +295,8 @@ void preload_update() {
   touch(k_leapfrog_f64);
   touch(k_pack);
   touch(k_pack_f64);
+  touch(k_check_state);
+  touch(k_check_state_f64);
   touch(k_scatter1);
   touch(k_scatter1_f64);
   touch(k_scatter3);

@@ -226,6 +226,17 @@ class NBody:
         self._ck(self.lib.nbody_get_state(self.h, _ptr(pm), _ptr(vi)))
         return pm, vi
 
+    def set_state(self, pos_m, vel_id, steps: int = 0):
+        """Checkpoint restore (nbody_set_state / nbody_set_state64): the slot-order
+        state of get_state() / get_state64() with its ids, and the step counter
+        (stats()["steps"] of the checkpointed context)."""
+        if self.precision == 64:
+            p, v = _f64(pos_m, self.n, 4), _f64(vel_id, self.n, 4)
+            self._ck(self.lib.nbody_set_state64(self.h, _ptr(p), _ptr(v), int(steps)))
+            return
+        p, v = _f32(pos_m, self.n, 4), _f32(vel_id, self.n, 4)
+        self._ck(self.lib.nbody_set_state(self.h, _ptr(p), _ptr(v), int(steps)))
+
     def stats(self) -> dict:
         s = _capi.nbody_stats()
         self._ck(self.lib.nbody_get_stats(self.h, C.byref(s)))
