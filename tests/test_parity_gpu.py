@@ -244,14 +244,14 @@ def test_invalid_bodies_rejected(NB):
 
 
 # ---------------------------------------------------------------- full size --
-def _sampled_full_size(NB, oracle, name, n, seed, nsample):
+def _sampled_full_size(NB, oracle, name, n, seed, nsample, theta=0.5):
     pos, vel, mass = generate(name, n, seed)
-    sim = NB(n, 0.5, EPS, DT, key_bits=16)
+    sim = NB(n, theta, EPS, DT, key_bits=16)
     sim.set_bodies(pos, vel, mass)
     sim.compute_accel()
     rng = np.random.default_rng(seed)
     targets = np.sort(rng.choice(n, nsample, replace=False))
-    ref = oracle.step(pos, vel, mass, theta=0.5, eps=EPS, dt=DT, key_bits=16, integrate=False, targets=targets)
+    ref = oracle.step(pos, vel, mass, theta=theta, eps=EPS, dt=DT, key_bits=16, integrate=False, targets=targets)
     assert (sim.debug_keys() == ref.keys).all()
     assert (sim.debug_perm() == ref.perm).all()
     # node records: the top 8 levels entirely, sampled nodes below
@@ -275,6 +275,17 @@ def test_config2_plummer_1M_sampled(NB, oracle):
 @pytest.mark.slow
 def test_config3_disks_10M_sampled(NB, oracle):
     _sampled_full_size(NB, oracle, "disks", 10_000_000, 3, 2000)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,seed,theta", [("uniform", 5, 0.3), ("clustered", 6, 0.8)])
+def test_config5_theta_sweep_10M_sampled(NB, oracle, name, seed, theta):
+    """Config 5 (theta sweep at N = 10^7, uniform vs clustered) at its two
+    extremes: the narrowest opening angle on the uniform cube (longest lists)
+    and the widest on the clustered set (accepted nodes may contain the
+    target, [A4]); keys, permutation, node records, counts and sampled
+    accelerations against the oracle."""
+    _sampled_full_size(NB, oracle, name, 10_000_000, seed, 1000, theta=theta)
 
 
 @pytest.mark.slow
