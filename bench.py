@@ -380,8 +380,21 @@ def run_ours(args, cfg, world, rank, local):
     if args.sort_every != 1:
         sim.set_option(7, args.sort_every)  # NBODY_OPT_SORT_EVERY
         cfg["sort_every"] = args.sort_every
+    use_peer = world > 1 and args.exchange == "peer" and world <= 8
+    if use_peer and not one_device:
+        # every rank must reach every other rank's GPU by loads/stores (NVLink /
+        # NVSwitch P2P); decided collectively so that all ranks pick the same
+        # exchange, else the NCCL all-gather on torch's communicator
+        devs = [None] * world
+        dist.all_gather_object(devs, local)
+        ok = all(d == local or torch.cuda.can_device_access_peer(local, d) for d in devs)
+        flag = torch.tensor([1 if ok else 0], device="cuda")
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if not int(flag.item()):
+            use_peer = False
+            cfg["exchange_note"] = "no peer access between the ranks' GPUs: NCCL all-gather instead"
     if world > 1:
-        if args.exchange == "peer" and world <= 8:
+        if use_peer:
             sim.attach_peers_group(rank, world)
             if args.balance == "cost":
                 sim.set_option(9, 1)  # NBODY_OPT_BALANCE
