@@ -53,6 +53,22 @@ def nccl_dir():
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
+    # several processes (torchrun ranks, pytest workers) may find the library
+    # stale at once: one builds under an exclusive lock, the others wait and
+    # then find it fresh; the result is written under a per-process name and
+    # renamed into place atomically
+    import fcntl
+    with open(LIB + ".lock", "w") as lock:
+        fcntl.flock(lock, fcntl.LOCK_EX)
+        try:
+            if not force and not stale():
+                return LIB
+            return _build_locked(verbose)
+        finally:
+            fcntl.flock(lock, fcntl.LOCK_UN)
+
+
+def _build_locked(verbose: bool) -> str:
     nccl = []
     d = nccl_dir()
     if d:
@@ -61,13 +77,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
         nccl = ["-DNBODY_WITH_NCCL", "-I", os.path.join(d, "include"), "-L", lib, f"-l:{so[0]}",
                 "-Xlinker", f"-rpath,{lib}"]
     extra = os.environ.get("NBODY_NVCC_FLAGS", "").split()  # tuning experiments only
+    tmp = f"{LIB}.{os.getpid()}.tmp"
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-I", os.path.join(ROOT, "include"), *nccl, *extra, "-o", LIB + ".tmp", *sources()]
+           "-I", os.path.join(ROOT, "include"), *nccl, *extra, "-o", tmp, *sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), file=sys.stderr)
     subprocess.run(cmd, check=True)
-    os.replace(LIB + ".tmp", LIB)
+    os.replace(tmp, LIB)
     return LIB
 
 

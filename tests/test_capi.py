@@ -106,3 +106,24 @@ def test_workspace_bytes_host_side(lib):
     h = C.c_void_p()
     assert lib.nbody_create_ws(10, 0.5, 1e-3, 1e-3, None, 1 << 20, C.byref(h)) == -1 and not h.value
     assert lib.nbody_attach_comm(None, None, 0, 1) == -1
+
+
+def test_concurrent_builds_do_not_race(tmp_path):
+    """torchrun ranks (or test workers) that find the library stale at the
+    same time: one process compiles under the build lock, the other waits and
+    loads the result; neither fails on the other's temporary file."""
+    import sys
+    import textwrap
+    lib = str(tmp_path / "libnbody_race.so")
+    code = textwrap.dedent(f"""
+        import sys
+        sys.path.insert(0, {ROOT!r})
+        from paper_conf_sc_casselldahg24_b200 import build as B
+        B.LIB = {lib!r}
+        B.build()
+        import ctypes
+        ctypes.CDLL(B.LIB).nbody_version
+    """)
+    procs = [subprocess.Popen([sys.executable, "-c", code]) for _ in range(2)]
+    assert [p.wait(timeout=900) for p in procs] == [0, 0]
+    assert os.path.exists(lib) and not [f for f in os.listdir(tmp_path) if f.endswith(".tmp")]

@@ -120,6 +120,40 @@ def test_zero_softening_with_coincident_pairs(NB, oracle):
     _check_pass(NB, oracle, pos, vel, mass, theta=0.5, eps=0.0)
 
 
+@pytest.mark.parametrize("scale,offset,eps", [(1e3, 5e3, 1.0), (1e-12, 2e-12, 1e-15), (1e6, -3e6, 1e3),
+                                              (1.0, 0.0, 1e-3)])
+def test_translated_and_scaled_inputs(NB, oracle, scale, offset, eps):
+    """The fp32 filters' error bounds carry the coordinate range R (DESIGN.md
+    "fp32 filter", "T filter"): translated, tiny and huge coordinates must
+    still give exactly the oracle's keys, trees and interaction lists
+    (undecided cases fall back to the fp64 test)."""
+    pos, vel, mass = generate("disks", 12_007, 12)
+    pos = (pos.astype(np.float64) * scale + offset).astype(np.float32)
+    _check_pass(NB, oracle, pos, vel, mass, theta=0.5, eps=eps)
+
+
+def test_far_offset_keeps_the_lists(NB, oracle):
+    """Coordinates 10^4 times the system size away from the origin: the fp32
+    state then resolves the near field only to ~1e-3 of a body spacing, so
+    fp32 monopoles (c32) may differ from the oracle's fp64 ones beyond the
+    force tolerance, but every opening decision -- hence every list and
+    count -- is still the oracle's (the filters widen with R)."""
+    pos, vel, mass = generate("disks", 12_007, 14)
+    pos = (pos.astype(np.float64) + 1e4).astype(np.float32)
+    sim = _run_gpu(NB, pos, vel, mass, 0.5, 16)
+    ref = oracle.step(pos, vel, mass, theta=0.5, eps=EPS, dt=DT, key_bits=16, integrate=False)
+    assert (sim.debug_keys() == ref.keys).all() and (sim.debug_perm() == ref.perm).all()
+    assert (sim.get_interactions()[ref.ids] == ref.count).all()
+
+
+@pytest.mark.parametrize("theta", [1.2, 4.0])
+def test_wide_opening_angles(NB, oracle, theta):
+    """theta beyond 1/sqrt(3): an accepted node may contain the target [A4]
+    (no special case on either side); lists and counts still equal."""
+    pos, vel, mass = generate("plummer", 9_001, 13)
+    _check_pass(NB, oracle, pos, vel, mass, theta=theta)
+
+
 def test_mixed_masses(NB, oracle):
     pos, vel, _ = generate("clustered", 8000, 9)
     mass = np.random.default_rng(9).lognormal(0.0, 1.0, 8000).astype(np.float32)
