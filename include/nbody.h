@@ -187,7 +187,9 @@ nbody_status nbody_set_option(nbody_ctx *ctx, int option, int64_t value);
 /* Load the bodies: pos[n][3], vel[n][3] (read as v_{-1/2} [A14]), mass[n],
  * fp32, host or device.  Copies them; resets slot order to array order and
  * ids to array indices.  Masses must be > 0 and finite, positions and
- * velocities finite [A18]. */
+ * velocities finite [A18].  The fp32 interaction forms m (r^2 + eps^2)^(-3/2)
+ * in fp32, so units must keep it (for the closest pairs) below ~3e38 [A15];
+ * the FP64 mode (NBODY_OPT_PRECISION = 64) has the fp64 range. */
 nbody_status nbody_set_bodies(nbody_ctx *ctx, const float *pos, const float *vel, const float *mass);
 /* NEXT-2 FP64 mode (NBODY_OPT_PRECISION = 64): as nbody_set_bodies with
  * fp64 pos[n][3], vel[n][3], mass[n] (host or device; copied).
