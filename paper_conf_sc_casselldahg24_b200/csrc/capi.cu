@@ -1739,7 +1739,8 @@ nbody_status nbody_debug_keys(nbody_ctx* c, uint64_t* keys) {
     return fail(c, NBODY_ENOMEM, "host buffer");
   }
   for (int64_t i = 0; i < n; ++i) wide[i] = tmp[i];
-  e = cudaMemcpy(keys, wide, 8 * size_t(n), cudaMemcpyDefault);
+  e = cudaMemcpyAsync(keys, wide, 8 * size_t(n), cudaMemcpyDefault, c->stream);  // stream-ordered, like every copy
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
   delete[] tmp;
   delete[] wide;
   if (e != cudaSuccess) return fail(c, NBODY_ECUDA, cudaGetErrorString(e));
