@@ -98,22 +98,27 @@ struct ForceParams {
   PeerTable xp{};
   // Super-group pre-pass (k_force.cu K6a): per super-group of kSG
   // consecutive owned targets, the nodes every one of them accepts (acc) and
-  // the frontier of nodes its box does not decide (fr); cnt = (n_acc, n_fr),
-  // (-1, -1) after an overflow (the warps then start from the root).
+  // the frontier of nodes its box does not decide (fr); cnt = (n_acc, n_fr)
+  // (the lists are bounded, never dropped; sg_cnt = null: no lists, the warps
+  // start from the root).
   uint32_t* sg_acc = nullptr;
   uint32_t* sg_fr = nullptr;
   int2* sg_cnt = nullptr;
 };
 
-// Super-group size and list capacities of K6a (k_force.cu).
+// Super-group size and list capacities of K6a (k_force.cu): 4096 accepted +
+// 2048 frontier ids per 256 targets (96 B per body).  Lists that would
+// overflow are cut short (the rest becomes frontier), never dropped; the
+// round-2 lists of 2048 + 1024 overflowed on 6 % of the clustered 10^8
+// super-groups and on nearly all at theta = 0.3 (profiles/r02_ab_k6.md).
 #ifndef NBODY_SG
 #define NBODY_SG 256
 #endif
 #ifndef NBODY_SG_ACC
-#define NBODY_SG_ACC 2048
+#define NBODY_SG_ACC 4096
 #endif
 #ifndef NBODY_SG_FR
-#define NBODY_SG_FR 1024
+#define NBODY_SG_FR 2048
 #endif
 constexpr int kSG = NBODY_SG, kSGAcc = NBODY_SG_ACC, kSGFr = NBODY_SG_FR;
 inline int64_t sg_groups(int64_t n) { return kSG > 0 ? (n + kSG - 1) / kSG + 1 : 0; }

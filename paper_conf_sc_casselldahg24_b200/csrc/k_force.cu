@@ -1413,6 +1413,20 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
   if (lane == 0) stk[0] = 1u;
   __syncwarp();
   while (na > 0) {
+    // Bounded lists (wide opening angles reach thousands of nodes per super-
+    // group): once the frontier could no longer take one more batch plus the
+    // whole stack, the stack itself becomes frontier and the walk stops; once
+    // the accepted list is full, accepted nodes go to the frontier too.  Every
+    // such node has only ancestors opened by all kSG targets, so the force
+    // warps continue from it exactly as from the root (their smaller boxes
+    // accept what this box accepts).  One batch adds <= 32 frontier entries
+    // and <= 64 - take stack entries, hence the margin of 96.
+    if (nfr + na + 96 > kSGFr) {
+      for (int i = lane; i < na; i += 32) fr[nfr + i] = stk[i];
+      nfr += na;
+      break;
+    }
+    const bool acc_full = nacc + 32 > kSGAcc;
     const int take = na < 32 ? na : 32;
     const int base = na - take;
     const bool has = lane < take;
@@ -1439,7 +1453,7 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
         const float dmin2 = fmaf(nz, nz, fmaf(ny, ny, nx * nx));
         const float dmax2 = fmaf(fz, fz, fmaf(fy, fy, fx * fx));
         if (dmin2 * (1.f - 4e-6f) > c.y) {
-          cls = 1;
+          cls = acc_full ? 3 : 1;
         } else if (dmax2 * (1.f + 4e-6f) < c.x && !guard) {
           cls = 2;
           const int l = L - 31 + __clz(int(g));
@@ -1450,17 +1464,10 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
       }
     }
     const uint32_t ba = __ballot_sync(kFull, cls == 1), bf = __ballot_sync(kFull, cls == 3);
-    if (cls == 1) {
-      const int pos = nacc + __popc(ba & lt);
-      if (pos < kSGAcc) acc[pos] = g;
-    }
-    if (cls == 3) {
-      const int pos = nfr + __popc(bf & lt);
-      if (pos < kSGFr) fr[pos] = g;
-    }
+    if (cls == 1) acc[nacc + __popc(ba & lt)] = g;
+    if (cls == 3) fr[nfr + __popc(bf & lt)] = g;
     nacc += __popc(ba);
     nfr += __popc(bf);
-    if (nacc > kSGAcc || nfr > kSGFr) break;  // overflow: the force warps start from the root
     const uint32_t b1 = __ballot_sync(kFull, cls == 2), b2 = __ballot_sync(kFull, cls == 2 && two);
     if (cls == 2) {
       const int pos = na + __popc(b1 & lt) + __popc(b2 & lt);
@@ -1470,8 +1477,7 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
     na += __popc(b1) + __popc(b2);
     __syncwarp();
   }
-  if (lane == 0)
-    P.sg_cnt[sgi] = (nacc > kSGAcc || nfr > kSGFr) ? make_int2(-1, -1) : make_int2(nacc, nfr);
+  if (lane == 0) P.sg_cnt[sgi] = make_int2(nacc, nfr);
 }
 
 }  // namespace

@@ -27,6 +27,8 @@ ap.add_argument("--n", type=int, default=10_000_000)
 ap.add_argument("--seed", type=int, default=3)
 ap.add_argument("--theta", type=float, default=0.5)
 ap.add_argument("--flags", default="")
+ap.add_argument("--no-build", action="store_true", help="reuse the stats library built by an earlier run")
+ap.add_argument("--json", default="", help="append one JSON record of the per-warp counters to this file")
 a = ap.parse_args()
 
 from paper_conf_sc_casselldahg24_b200 import build as B  # noqa: E402
@@ -34,7 +36,8 @@ from paper_conf_sc_casselldahg24_b200 import build as B  # noqa: E402
 lib = "/tmp/libnbody_b200_stats.so"
 os.environ["NBODY_NVCC_FLAGS"] = ("-DNBODY_K6_STATS " + a.flags).strip()
 B.LIB = lib
-B.build(force=True)
+if not (a.no_build and os.path.exists(lib)):
+    B.build(force=True)
 from paper_conf_sc_casselldahg24_b200 import _capi, NBody  # noqa: E402
 from workloads import generate  # noqa: E402
 
@@ -58,3 +61,11 @@ pl = v[7] / max(v[6], 1)
 print(f"  partial-entry lane use {pl:.2f}/32; full lanes share of interactions {v[8] / inter:.3f}; "
       f"partial lanes share {v[7] / inter:.3f}")
 print(f"  T nodes per batch {v[4] / max(v[3], 1):.1f}; A nodes per batch {v[2] / max(v[1], 1):.1f}")
+
+if a.json:
+    import json
+    rec = {"workload": a.workload, "n": a.n, "seed": a.seed, "theta": a.theta, "interactions": inter,
+           "warps": w, "per_warp": {name: x / w for name, x in zip(kStatNames, v)},
+           "partial_lane_use": pl, "dense_lane_util": (v[7] + v[8]) / max(32.0 * (v[5] + v[6]), 1.0)}
+    with open(a.json, "a") as f:
+        f.write(json.dumps(rec) + "\n")

@@ -38,7 +38,7 @@ for name, n, seed, theta, quad in [("disks", 40_000, 3, 0.5, False), ("clustered
     cnt = sim.get_interactions()[ref.ids]
     e = rel_errors(sim.get_accel()[ref.ids], ref.acc)
     out.append({"case": f"{name} n={n} theta={theta} quad={quad}", "stats_len": got,
-                "spill_walks": int(buf[14]), "guard_handovers": int(buf[36]),
+                "spill_walks": int(buf[14]), "guard_handovers": int(buf[36]), "no_sg_lists": int(buf[49]),
                 "counts_equal": bool((cnt == ref.count).all()), "lane_util": lane_util,
                 "rms": float(np.sqrt(np.mean(e ** 2))), "max": float(e.max())})
     sim.close()

@@ -23,15 +23,23 @@ pytestmark = pytest.mark.gpu
 HERE = os.path.dirname(os.path.abspath(__file__))
 
 
+TINY_K6 = ("-DNBODY_K6_STATS -DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 "
+           "-DNBODY_CAP_A=64 -DNBODY_QCAP_A=64 -DNBODY_QCAP_P=32 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64")
+# K6a's bounded super-group lists: 64 accepted ids and 160 frontier ids, so
+# every super-group fills its accepted list (the rest goes to the frontier)
+# and dumps its stack into the frontier early (wide lists, theta = 0.3)
+TINY_K6A = "-DNBODY_K6_STATS -DNBODY_SG_ACC=64 -DNBODY_SG_FR=160"
+
+
 @pytest.mark.timeout(900)
-def test_overflow_paths_match_the_oracle(tmp_path):
+@pytest.mark.parametrize("flags,overflow", [(TINY_K6, True), (TINY_K6A, False)], ids=["k6_caps", "k6a_lists"])
+def test_overflow_paths_match_the_oracle(tmp_path, flags, overflow):
     import torch
     assert torch.cuda.is_available()
     from paper_conf_sc_casselldahg24_b200 import build as B
     lib = str(tmp_path / "libnbody_smallcaps.so")
     env = dict(os.environ)
-    env["NBODY_NVCC_FLAGS"] = ("-DNBODY_K6_STATS -DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 "
-                               "-DNBODY_CAP_A=64 -DNBODY_QCAP_A=64 -DNBODY_QCAP_P=32 -DNBODY_QCAP_F=32 -DNBODY_QCAP_T=64")
+    env["NBODY_NVCC_FLAGS"] = flags
     code = f"from paper_conf_sc_casselldahg24_b200 import build as B; B.LIB = {lib!r}; B.build(force=True)"
     subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=os.path.dirname(HERE))
     env["NBODY_TEST_LIB"] = lib
@@ -47,7 +55,9 @@ def test_overflow_paths_match_the_oracle(tmp_path):
     assert sim.stats()["lane_util"] == -1.0  # the product build carries no counters
     for c in res:
         assert c["stats_len"] == 52, c
-        assert c["spill_walks"] > 0 and c["guard_handovers"] > 0, c
+        if overflow:
+            assert c["spill_walks"] > 0 and c["guard_handovers"] > 0, c
+        assert c["no_sg_lists"] == 0, c  # every warp starts from its super-group's lists
         assert c["counts_equal"], c
         assert 0.0 < c["lane_util"] <= 1.0, c  # nbody_get_stats reports the counters of a stats build
         assert c["rms"] <= ACC_RMS_TOL and c["max"] <= ACC_MAX_TOL, c
