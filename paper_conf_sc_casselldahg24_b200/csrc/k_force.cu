@@ -1105,8 +1105,11 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     if (na == 0 && S.sg_next < S.sg_nfr) {  // refill the box stack from the super-group frontier
       const int next = S.sg_next;
       const int take = min(S.sg_nfr - next, S.kA - 32);  // after a 32-node pop, room for 64 pushes
+      // each chunk is popped in list order (the super-group walk's discovery
+      // order: coarser nodes first), -0.5 % K6 against the reverse
+      // (profiles/r02_ab_k6.md)
       const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
-      for (int i = lane; i < take; i += 32) S.astk[i] = __ldg(fl + i);
+      for (int i = lane; i < take; i += 32) S.astk[take - 1 - i] = __ldg(fl + i);
       __syncwarp();
       if (lane == 0) S.sg_next = next + take;
       na = take;
