@@ -7,7 +7,10 @@ nodes to the transposed phase -- would then never run in a test.  Here the
 library is rebuilt with tiny capacities (T stack 64, dense lists 32, box
 stack 64) plus the event counters, so both paths run on every warp, and the
 results must still equal the oracle's: counts equal for every body,
-accelerations within the north-star tolerances.
+accelerations within the north-star tolerances.  A second build shrinks
+K6a's super-group lists instead, so that every list is cut short (accepted
+nodes spill into the frontier, the frontier takes the remaining stack) and
+the force warps must still reproduce the lists of the walk from the root.
 """
 import json
 import os
