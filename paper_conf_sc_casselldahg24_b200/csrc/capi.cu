@@ -186,7 +186,7 @@ constexpr int64_t kPartPad = 256 * kMaxWorld;  // G * S - N < 256 G
 // [A21] S = ceil(N / G) rounded up to a multiple of kPartUnit = 256 slots:
 // the warp groups (32) and K6a's super-groups (kSG = 256) then coincide
 // with the single-GPU run, so results are bit-identical.
-constexpr int64_t kPartUnit = 256;
+constexpr int64_t kPartUnit = kPartUnitSlots;
 static_assert(kSG <= 0 || kPartUnit % kSG == 0, "rank ranges must start at super-group boundaries");
 void set_part(nbody_ctx* c, int rank, int world) {
   const int64_t n = c->n;

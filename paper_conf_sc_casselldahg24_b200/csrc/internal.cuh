@@ -121,6 +121,9 @@ struct ForceParams {
 #define NBODY_SG_FR 2048
 #endif
 constexpr int kSG = NBODY_SG, kSGAcc = NBODY_SG_ACC, kSGFr = NBODY_SG_FR;
+// multi-GPU partition unit [A21]: rank ranges start at multiples of it, so
+// they start at super-group boundaries (256 slots, or kSG if larger)
+constexpr int kPartUnitSlots = kSG > 256 ? kSG : 256;
 inline int64_t sg_groups(int64_t n) { return kSG > 0 ? (n + kSG - 1) / kSG + 1 : 0; }
 
 // ---- K1 / K2 --------------------------------------------------------------

@@ -74,7 +74,7 @@ __global__ __launch_bounds__(256) void k_leapfrog_scatter(const float4* __restri
 // chunk of units, a block scan of the chunk sums locates the chunk holding
 // each target, whose thread walks it.
 constexpr int kPartThreads = 1024;
-constexpr int kUnitGroups = 8;  // 32-slot cost groups per 256-slot unit
+constexpr int kUnitGroups = kPartUnitSlots / 32;  // 32-slot cost groups per partition unit
 
 __device__ __forceinline__ unsigned long long unit_cost(const uint32_t* __restrict__ w, int64_t J, int64_t u) {
   unsigned long long c = 0;
