@@ -172,3 +172,24 @@ def test_resume_fp64_mode(NB):
     frac[0, 3] += 0.5                          # not an integer id
     with pytest.raises(NBodyError, match="permutation"):
         b.set_state(pm, frac, 2)
+
+
+def test_resume_with_quadrupoles_and_tree_reuse(NB):
+    """The restore carries everything a quadrupole, tree-reuse run needs: the
+    resumed context steps bit-identically (moments are rebuilt from the
+    restored state each step)."""
+    n = 15_013
+    pos, vel, mass = generate("clustered", n, 97)
+    a = NB(n, 0.6, EPS, DT, multipole=2)
+    a.set_option(7, 3)
+    a.set_bodies(pos, vel, mass)
+    a.step(4)
+    pm, vi = a.get_state()
+    steps = a.stats()["steps"]
+    a.step(3)
+    b = NB(n, 0.6, EPS, DT, multipole=2)
+    b.set_option(7, 3)
+    b.set_state(pm, vi, steps)
+    b.step(3)
+    assert (b.get_state()[0].view(np.uint32) == a.get_state()[0].view(np.uint32)).all()
+    assert (b.get_accel().view(np.uint32) == a.get_accel().view(np.uint32)).all()

@@ -444,6 +444,25 @@ def test_tree_reuse_against_oracle(NB, oracle):
         _check_update(pm1[:, :3], vi1[:, :3], r1, dt)
 
 
+def test_tree_reuse_with_quadrupoles_against_oracle(NB, oracle):
+    """NEXT-3(iii) with NEXT-4 [A23][A24]: a reuse step refits the second
+    moments too; on the reuse step's input state the oracle's
+    resort=False, quad=True step has the same lists and moments."""
+    n, dt = 20_000, 1e-3
+    pos, vel, mass = generate("clustered", n, 86)
+    s = NB(n, 0.6, EPS, dt, multipole=2)
+    s.set_option(7, 2)
+    s.set_bodies(pos, vel, mass)
+    s.step(1)
+    pm, vi = s.get_state()
+    ids0 = vi[:, 3].view(np.int32).copy()
+    s.step(1)  # reuse step
+    r1 = oracle.step(pm[:, :3], vi[:, :3], pm[:, 3], ids0, theta=0.6, eps=EPS, dt=dt, resort=False, quad=True)
+    assert (r1.ids == ids0).all()
+    assert (s.get_interactions()[r1.ids] == r1.count).all()
+    assert_acc_close(s.get_accel()[r1.ids], r1.acc)
+
+
 def _check_update(x_gpu, v_gpu, ref, dt=DT):
     """Leapfrog O8 on the same input: v = v0 + a dt, x = x0 + v dt with the
     GPU's fp32 a (within the acceleration tolerance) -- differences are
