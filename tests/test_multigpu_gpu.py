@@ -441,3 +441,29 @@ def test_emulated_partition_matches_oracle_each_step(NB, oracle, world, n):
         assert covered.all()     # the owned slices cover every body exactly once between them
         pm, vi = _oracle_gate(oracle, ranks, ref, owned)
         x, v, m, ids = pm[:, :3], vi[:, :3], pm[:, 3], vi[:, 3].view(np.int32).copy()
+
+
+@pytest.mark.parametrize("world,kw", [(2, {}), (4, {"balance": True})])
+def test_peer_exchange_resumes_from_a_checkpoint(NB, world, kw):
+    """Checkpoint / resume across the exchange: every rank restores the same
+    slot-order state (nbody_set_state) and the G-rank run continues bit-
+    identically to the uninterrupted one-GPU run."""
+    n = 12_011
+    pos, vel, mass = generate("disks", n, 71)
+    ref = NB(n, 0.5, 1e-3, 1e-3)
+    ref.set_bodies(pos, vel, mass)
+    ref.step(2)
+    pm, vi = ref.get_state()
+    ref.step(2)
+    x_ref, a_ref = ref.get_positions(), ref.get_accel()
+    ranks = [NB(n, 0.5, 1e-3, 1e-3, **kw) for _ in range(world)]
+    NB.attach_peers_local(ranks)
+    for s in ranks:
+        s.set_state(pm, vi, 2)
+    for _ in range(2):
+        for s in ranks:
+            s.step(1)
+    for s in ranks:
+        s.sync()
+        assert (s.get_positions() == x_ref).all()
+        assert (s.get_accel() == a_ref).all()
