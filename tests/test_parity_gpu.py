@@ -156,6 +156,17 @@ def test_wide_opening_angles(NB, oracle, theta):
     _check_pass(NB, oracle, pos, vel, mass, theta=theta)
 
 
+def test_dominant_central_mass(NB, oracle):
+    """A galaxy with a central mass 10^6 times the others (node COMs pulled
+    onto one body, masses spanning 6 decades in the fp64 moments and the
+    fp32 records): records bit-exact, lists equal, accelerations in tolerance."""
+    pos, vel, mass = generate("plummer", 10_001, 15)
+    pos[0] = 0.0
+    mass = mass.copy()
+    mass[0] = mass[1] * 1e6
+    _check_pass(NB, oracle, pos, vel, mass, theta=0.5)
+
+
 def test_mixed_masses(NB, oracle):
     pos, vel, _ = generate("clustered", 8000, 9)
     mass = np.random.default_rng(9).lognormal(0.0, 1.0, 8000).astype(np.float32)
