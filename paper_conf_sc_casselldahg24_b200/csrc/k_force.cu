@@ -1102,17 +1102,23 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
     }
   }
   while (true) {
-    if (na == 0 && S.sg_next < S.sg_nfr) {  // refill the box stack from the super-group frontier
+    // Refill the box stack from the super-group frontier whenever it holds
+    // less than one batch (the chunk goes below the nodes still stacked, so
+    // box batches stay full); each chunk is popped in list order (the super-
+    // group walk's discovery order, coarser nodes first): -0.5 % and -0.2 %
+    // K6 against refilling an empty stack popped from the chunk's end
+    // (profiles/r02_ab_k6.md).
+    if (na < 32 && S.sg_next < S.sg_nfr) {
       const int next = S.sg_next;
-      const int take = min(S.sg_nfr - next, S.kA - 32);  // after a 32-node pop, room for 64 pushes
-      // each chunk is popped in list order (the super-group walk's discovery
-      // order: coarser nodes first), -0.5 % K6 against the reverse
-      // (profiles/r02_ab_k6.md)
+      const int take = min(S.sg_nfr - next, S.kA - 32 - na);  // after a 32-node pop, room for 64 pushes
+      const uint32_t keep = lane < na ? S.astk[lane] : 0u;
+      __syncwarp();
+      if (lane < na) S.astk[take + lane] = keep;
       const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
       for (int i = lane; i < take; i += 32) S.astk[take - 1 - i] = __ldg(fl + i);
       __syncwarp();
       if (lane == 0) S.sg_next = next + take;
-      na = take;
+      na += take;
     }
     if (nt >= 32 || (na == 0 && nt > 0)) {
       // ---- T: transposed classification of up to 32 (node, mask) entries
