@@ -59,6 +59,23 @@
 
 #include "internal.cuh"
 
+// Design/debug build (-DNBODY_DEBUG_BOUNDS): device-side bounds checks on
+// every list and stack write of K6 and K6a (a failed check traps the kernel);
+// the stand-in for compute-sanitizer memcheck, which the GPU pool no longer
+// offers (tests/test_small_caps_gpu.py runs the tiny-capacity builds with it).
+#ifdef NBODY_DEBUG_BOUNDS
+#include <cstdio>
+#define NB_CHECK(cond)                                                                              \
+  do {                                                                                              \
+    if (!(cond)) {                                                                                  \
+      printf("NB_CHECK failed: %s (%s:%d)\n", #cond, __FILE__, __LINE__);                            \
+      __trap();                                                                                     \
+    }                                                                                               \
+  } while (0)
+#else
+#define NB_CHECK(cond) ((void)0)
+#endif
+
 namespace nb {
 
 // Traversal event counters for design work (NBODY_K6_STATS builds only;
@@ -994,6 +1011,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       if constexpr (kF64)
         S.frec64[pos] = P.t.rec64[g];
       else
+        NB_CHECK(pos < S.kF);
         S.frec[pos >> 1].put(pos & 1, r);
       if constexpr (kQuad) S.fq[pos >> 1].put(pos & 1, q0, q1);
     }
@@ -1003,6 +1021,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
         S.prec64[pos] = P.t.rec64[g];
       else
         S.prec[pos >> 1].put(pos & 1, r);
+      NB_CHECK(pos < S.kP);
       S.pmsk[pos] = msk;
       if constexpr (kQuad) S.pq[pos >> 1].put(pos & 1, q0, q1);
     }
@@ -1113,6 +1132,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       const int take = min(S.sg_nfr - next, S.kA - 32 - na);  // after a 32-node pop, room for 64 pushes
       const uint32_t keep = lane < na ? S.astk[lane] : 0u;
       __syncwarp();
+      NB_CHECK(take + na <= S.kA);
       if (lane < na) S.astk[take + lane] = keep;
       const uint32_t* fl = P.sg_fr + size_t(sgi) * kSGFr + next;
       for (int i = lane; i < take; i += 32) S.astk[take - 1 - i] = __ldg(fl + i);
@@ -1246,6 +1266,7 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       const uint32_t b2 = __ballot_sync(kFull, push && two);
       if (push) {
         const int pos = nt + __popc(b1 & lt) + __popc(b2 & lt);
+        NB_CHECK(pos + int(two) < S.kT);
         S.tstk[pos] = make_uint2(2u * g, rm);
         if (two) S.tstk[pos + 1] = make_uint2(2u * g + 1u, rm);
       }
@@ -1346,12 +1367,14 @@ __global__ __launch_bounds__(32 * kV0Warps, kF64 ? NBODY_V0_MINB_F64 : NBODY_V0_
       if (cls == 1 && g >= leaf0 && g - kid0 < 32u) msk &= ~(1u << (g - kid0));  // not on itself
       append(cls == 1, r, msk, g < leaf0 ? g : 0u, g);
       const uint32_t bt = __ballot_sync(kFull, cls == 3);
+      if (cls == 3) NB_CHECK(nt + __popc(bt & lt) < S.kT);
       if (cls == 3) S.tstk[nt + __popc(bt & lt)] = make_uint2(g, amask);
       nt += __popc(bt);
       const uint32_t b1 = __ballot_sync(kFull, cls == 2);
       const uint32_t b2 = __ballot_sync(kFull, cls == 2 && two);
       if (cls == 2) {
         const int pos = na + __popc(b1 & lt) + __popc(b2 & lt);
+        NB_CHECK(pos + int(two) < S.kA);
         S.astk[pos] = 2u * g;
         if (two) S.astk[pos + 1] = 2u * g + 1u;
       }
@@ -1431,6 +1454,7 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
     // accept what this box accepts).  One batch adds <= 32 frontier entries
     // and <= 64 - take stack entries, hence the margin of 96.
     if (nfr + na + 96 > kSGFr) {
+      NB_CHECK(nfr + na <= kSGFr);
       for (int i = lane; i < na; i += 32) fr[nfr + i] = stk[i];
       nfr += na;
       break;
@@ -1473,6 +1497,8 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
       }
     }
     const uint32_t ba = __ballot_sync(kFull, cls == 1), bf = __ballot_sync(kFull, cls == 3);
+    if (cls == 1) NB_CHECK(nacc + __popc(ba & lt) < kSGAcc);
+    if (cls == 3) NB_CHECK(nfr + __popc(bf & lt) < kSGFr);
     if (cls == 1) acc[nacc + __popc(ba & lt)] = g;
     if (cls == 3) fr[nfr + __popc(bf & lt)] = g;
     nacc += __popc(ba);
@@ -1480,6 +1506,7 @@ __global__ __launch_bounds__(32 * kSGWarps) void k_force_sgroups(const ForcePara
     const uint32_t b1 = __ballot_sync(kFull, cls == 2), b2 = __ballot_sync(kFull, cls == 2 && two);
     if (cls == 2) {
       const int pos = na + __popc(b1 & lt) + __popc(b2 & lt);
+      NB_CHECK(pos + int(two) < kCapA);
       stk[pos] = 2u * g;
       if (two) stk[pos + 1] = 2u * g + 1u;
     }

@@ -32,10 +32,18 @@ TINY_K6 = ("-DNBODY_K6_STATS -DNBODY_CAP_T=64 -DNBODY_CAP_F=32 -DNBODY_CAP_P=32 
 # every super-group fills its accepted list (the rest goes to the frontier)
 # and dumps its stack into the frontier early (wide lists, theta = 0.3)
 TINY_K6A = "-DNBODY_K6_STATS -DNBODY_SG_ACC=64 -DNBODY_SG_FR=160"
+# every build here also carries the device-side bounds checks of every K6 /
+# K6a list and stack write (NB_CHECK in k_force.cu: a violation traps the
+# kernel and fails the worker) -- the stand-in for compute-sanitizer
+# memcheck, which the GPU pool no longer offers; the third build checks the
+# product capacities
+BOUNDS = " -DNBODY_DEBUG_BOUNDS"
 
 
 @pytest.mark.timeout(900)
-@pytest.mark.parametrize("flags,overflow", [(TINY_K6, True), (TINY_K6A, False)], ids=["k6_caps", "k6a_lists"])
+@pytest.mark.parametrize("flags,overflow", [(TINY_K6 + BOUNDS, True), (TINY_K6A + BOUNDS, False),
+                                            ("-DNBODY_K6_STATS" + BOUNDS, False)],
+                         ids=["k6_caps", "k6a_lists", "product_caps"])
 def test_overflow_paths_match_the_oracle(tmp_path, flags, overflow):
     import torch
     assert torch.cuda.is_available()
